@@ -1,0 +1,395 @@
+"""Benchmark: sequence evaluations/s of the parallel-SA hot path at n=1000 on B200 (BASELINE.json).
+
+One bench "step" = one pass of the whole hot path over BASELINE config 5 on this GPU: for each of
+the four CDD n=1000 instances (seed 1, h in {0.2,0.4,0.6,0.8}) the T0 rule (5000 random
+sequences), then 65,536 asynchronous SA chains x 5000 iterations (Alg. 1, P:194-198,
+mu=0.88, Pert=4 FY moves), then the reduction to the best -- and, on N>1 GPUs, the
+NCCL MIN all-reduce of the packed best plus the winner broadcast.  value = all sequence
+evaluations of all ranks / max-over-ranks device time.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl reference]
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+N_JOBS = 1000
+CHAINS = 65536
+SA_STEPS = 5000
+T0_SAMPLES = 5000
+HS = (0.2, 0.4, 0.6, 0.8)
+INSTANCE_SEED = 1
+RUN_SEED = 0x5EED0005
+METRIC = "sequence evals/s at n=1000 on 1/8 B200; SA % gap vs best-known"
+WORKLOAD = "config5: CDD n=1000, h in {0.2,0.4,0.6,0.8} (instance seed 1), 65536 SA chains/GPU x 5000 steps, T0 from 5000 samples"
+INT_OPS_PER_ELEM = 6  # 3 prefix adds + subtract + select + multiply-add per job
+
+
+def _peaks():
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:
+        return {}
+
+
+def _evals_per_step(chains, steps, samples, instances):
+    return instances * (samples + chains * (steps + 1))
+
+
+class ClockSampler:
+    """nvidia-smi clocks and throttle reasons sampled during the timed region."""
+
+    def __init__(self, index=0):
+        self.index = index
+        self.proc = None
+        self.lines = []
+
+    def __enter__(self):
+        q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+             "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+             "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", f"--id={self.index}", f"--query-gpu={q}", "--format=csv,noheader,nounits",
+                 "-lms", "200"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def __exit__(self, *a):
+        if self.proc is not None:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 8:
+                continue
+            try:
+                sm.append(float(f[0]))
+                mx = float(f[1])
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[4:8]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": mx,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ------------------------------------------------------------------------------ reference arm
+def run_reference(args):
+    """The CPU oracle (oracle/, untuned) on the box's host cores: a bounded sample of the same
+    workload (a few chains x steps of the same instances), same metric and unit."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    import gen
+    import oracle
+
+    threads = os.cpu_count() or 1
+    chains_per_thread, steps = 1, 400
+    insts = [oracle.Problem.from_instance(gen.cdd_instance(N_JOBS, INSTANCE_SEED, h)) for h in HS]
+    T0s = [oracle.t0(pr, oracle.CDD, RUN_SEED, 200) for pr in insts]
+
+    def one_step():
+        t = time.perf_counter()
+        for pr, T0 in zip(insts, T0s):
+            def work(tid):
+                p = oracle.sa_params(chains=chains_per_thread, steps=steps, seed=RUN_SEED,
+                                     chain_offset=tid * chains_per_thread)
+                oracle.sa_run(pr, p, T0)
+            ts = [threading.Thread(target=work, args=(i,)) for i in range(threads)]
+            [x.start() for x in ts]
+            [x.join() for x in ts]
+        return time.perf_counter() - t
+
+    for _ in range(args.warmup):
+        one_step()
+    dts = [one_step() for _ in range(args.steps)]
+    evals = len(HS) * threads * chains_per_thread * (steps + 1)
+    value = evals * args.steps / sum(dts)
+    sample = (f"{len(HS)} instances x {threads} threads x {chains_per_thread} chain x {steps} SA "
+              f"steps per bench step (T0 from 200 samples, excluded)")
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": "evals/s",
+            "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": 1000 * sum(dts) / args.steps, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "int32", "data": "synthetic",
+            "config": {"workload": WORKLOAD, "sample": sample},
+            "cpu_baseline": {"value": value, "unit": "evals/s", "cores": threads, "kind": "oracle",
+                             "sample": sample},
+            "e2e": {"value": value, "unit": "evals/s", "h2d_bytes_per_step": 0,
+                    "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def cpu_baseline_sample(seconds=12.0):
+    """Oracle SA timed on the host cores (bounded sample of the same workload)."""
+    import gen
+    import oracle
+
+    threads = os.cpu_count() or 1
+    pr = oracle.Problem.from_instance(gen.cdd_instance(N_JOBS, INSTANCE_SEED, 0.4))
+    T0 = oracle.t0(pr, oracle.CDD, RUN_SEED, 200)
+    # size the per-thread chain so the sample takes about `seconds`
+    t = time.perf_counter()
+    oracle.sa_chain(pr, oracle.sa_params(steps=200, seed=RUN_SEED), T0, 0)
+    per_eval = (time.perf_counter() - t) / 201
+    steps = max(50, int(seconds / per_eval))
+    done = [0]
+
+    def work(tid):
+        oracle.sa_chain(pr, oracle.sa_params(steps=steps, seed=RUN_SEED), T0, tid)
+        done[0] += steps + 1
+
+    ts = [threading.Thread(target=work, args=(i,)) for i in range(threads)]
+    t = time.perf_counter()
+    [x.start() for x in ts]
+    [x.join() for x in ts]
+    dt = time.perf_counter() - t
+    return {"value": done[0] / dt, "unit": "evals/s", "cores": threads, "kind": "oracle",
+            "sample": f"{threads} host threads x 1 SA chain x {steps} steps, CDD n=1000 h=0.4 "
+                      f"(T0 from 200 samples, excluded); {dt:.1f} s"}
+
+
+# ------------------------------------------------------------------------------ GPU arm
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=3)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--chains", type=int, default=CHAINS)
+    ap.add_argument("--sa-steps", type=int, default=SA_STEPS)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-eval", action="store_true")
+    args = ap.parse_args()
+    if args.impl == "reference":
+        return run_reference(args)
+
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    import gen
+    import paper_conf_ipps_awasthillw16_b200 as lib
+    from paper_conf_ipps_awasthillw16_b200 import dist as cdist
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    dev = torch.device("cuda", local)
+    stream = torch.cuda.current_stream(dev)
+
+    chains, steps = args.chains, args.sa_steps
+    gens = [gen.cdd_instance(N_JOBS, INSTANCE_SEED, h) for h in HS]
+    insts = [lib.Instance.from_gen(g, device=local) for g in gens]
+    ws = {}
+    T0buf = [torch.empty(1, dtype=torch.float64, device=dev) for _ in insts]
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    kernel_ev = []
+
+    def one_step(record=False):
+        out = []
+        for i, ins in enumerate(insts):
+            flush.fill_(i)  # L2 flush between instances (256 MiB write)
+            T0 = lib.sa_t0(ins, "cdd", seed=RUN_SEED, samples=T0_SAMPLES)
+            e1 = torch.cuda.Event(enable_timing=True)
+            e2 = torch.cuda.Event(enable_timing=True)
+            e1.record(stream)
+            r = lib.sa_run(ins, chains, steps, seed=RUN_SEED, chain_offset=rank * chains,
+                           T0_dev=T0, workspace=ws.get(i))
+            e2.record(stream)
+            ws[i] = r["workspace"]
+            if record:
+                kernel_ev.append((e1, e2))
+            if world > 1:
+                cdist.global_best(ins, chains)
+            out.append(ins)
+        return out
+
+    for _ in range(args.warmup):
+        one_step()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    with ClockSampler(local) as clk:
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        t0 = torch.cuda.Event(enable_timing=True)
+        t1 = torch.cuda.Event(enable_timing=True)
+        t0.record(stream)
+        for _ in range(args.steps):
+            one_step(record=True)
+        t1.record(stream)
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+    ms = t0.elapsed_time(t1)
+    if world > 1:
+        tt = torch.tensor([ms], device=dev, dtype=torch.float64)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        ms = float(tt.item())
+    evals = _evals_per_step(chains, steps, T0_SAMPLES, len(insts)) * args.steps * world
+    value = evals / (ms / 1000.0)
+
+    # quality: best of the last step per instance vs the oracle-made best-known values
+    gaps = {}
+    bk_path = os.path.join(ROOT, "tests", "golden", "best_known_n1000.json")
+    bk = json.load(open(bk_path)) if os.path.exists(bk_path) else {}
+    for g, ins in zip(gens, insts):
+        pen, perm, gid = lib.best_get(ins)
+        key = f"{g.h:.1f}"
+        entry = {"best": pen, "chain": gid}
+        if key in bk.get("best_known", {}):
+            ref = bk["best_known"][key]
+            entry["best_known"] = ref
+            entry["gap_pct"] = 100.0 * (pen - ref) / ref
+        gaps[key] = entry
+
+    # roofline of the dominant kernel (sa_kernel): algorithmic int ops / its event duration
+    peaks = _peaks()
+    sm_max = float(peaks.get("sm_max_mhz", 1965.0))
+    kms = [a.elapsed_time(b) for a, b in kernel_ev]
+    k_avg_ms = sum(kms) / len(kms)
+    ops = INT_OPS_PER_ELEM * N_JOBS * chains * (steps + 1)
+    achieved = ops / (k_avg_ms / 1000.0) / 1e12
+    nsm = torch.cuda.get_device_properties(dev).multi_processor_count
+    peak = 128 * nsm * sm_max * 1e6 / 1e12
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "sa_kernel_dram_bytes.json")
+    if os.path.exists(tp):
+        traffic = json.load(open(tp)).get("dram_bytes_per_launch")
+    step_ms = ms / args.steps
+    roofline = {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "Tint-op/s",
+                "frac": achieved / peak, "traffic": traffic, "kernel": "sa_kernel<32,cdd>",
+                "kernel_ms_avg": k_avg_ms, "kernel_share_of_step": k_avg_ms * len(insts) / step_ms,
+                "ops_per_launch": ops,
+                "peak_note": f"128 int32 lane-ops/clk/SM (4 SMSP x 32 lanes issue, alu+fma pipes) x {nsm} SMs x {sm_max:.0f} MHz max clock"}
+
+    extra = {}
+    if rank == 0 and not args.no_eval:
+        extra["eval_batch"] = bench_eval(lib, gens[1], dev, stream, peaks)
+    e2e = None
+    if not args.no_e2e:
+        e2e = bench_e2e(lib, gens, chains, steps, rank, world, dev, stream, max(1, args.steps // 2))
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cpu = cpu_baseline_sample()
+
+    if rank == 0:
+        line = {"metric": METRIC, "value": value, "unit": "evals/s", "n_gpus": world,
+                "steps": args.steps, "warmup": args.warmup, "ms_per_step": step_ms,
+                "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+                "dtype": "int32", "data": "synthetic",
+                "config": {"workload": WORKLOAD, "n": N_JOBS, "chains_per_gpu": chains,
+                           "sa_steps": steps, "t0_samples": T0_SAMPLES, "instances": len(insts),
+                           "parallelism": f"dp{world} (independent chains, NCCL min-allreduce)",
+                           "l2": "state is on-chip; L2 flushed (256 MiB write) before every instance"},
+                "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
+                "gpu_launches": 4 * len(insts) * args.steps,
+                "clocks": clk.summary(), "quality": gaps, **extra,
+                "context": {"paper_gpu": "GeForce GT 560M", "paper_sa_evals_per_s_n1000": 2.22e5,
+                            "paper_headline_speedup": "100x vs CPU [7] within 2% (P:7)"}}
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def bench_eval(lib, g, dev, stream, peaks, batch=1 << 20, reps=20):
+    """Batched evaluation kernel at n=1000 (HBM roofline), inputs 2 GiB >> L2."""
+    import torch
+
+    import gen
+
+    ins = lib.Instance.from_gen(g, device=dev.index)
+    pools = [gen.random_perms_device(batch, N_JOBS, 7 + i, device=dev) for i in range(2)]
+    out = torch.empty(batch, dtype=torch.int64, device=dev)
+    for i in range(3):
+        lib.cdd_eval_batch(ins, pools[i % 2], out)
+    torch.cuda.synchronize()
+    e1 = torch.cuda.Event(enable_timing=True)
+    e2 = torch.cuda.Event(enable_timing=True)
+    e1.record(stream)
+    for i in range(reps):
+        lib.cdd_eval_batch(ins, pools[i % 2], out)
+    e2.record(stream)
+    torch.cuda.synchronize()
+    ms = e1.elapsed_time(e2) / reps
+    lib.cdd_check(ins)
+    bytes_per = batch * (2 * N_JOBS + 8)
+    gbs = bytes_per / (ms / 1000) / 1e9
+    hbm = float(peaks.get("hbm_gbs", 6454.0))
+    return {"workload": "cdd_eval_batch, CDD n=1000 h=0.4, 2^20 random sequences (2 GiB, alternating pools > L2)",
+            "evals_per_s": batch / (ms / 1000), "ms_per_launch": ms,
+            "roofline": {"bound": "hbm", "achieved": gbs, "peak": hbm, "unit": "GB/s",
+                         "frac": gbs / hbm, "traffic": None,
+                         "algorithmic_bytes_per_eval": 2 * N_JOBS + 8}}
+
+
+def bench_e2e(lib, gens, chains, steps, rank, world, dev, stream, k):
+    """Same metric through the public API with HOST buffers: instance upload, SA, best download."""
+    import torch
+
+    from paper_conf_ipps_awasthillw16_b200 import dist as cdist
+
+    def step():
+        h2d = d2h = 0
+        for g in gens:
+            ins = lib.Instance(g.P, g.alpha, g.beta, g.d, device=dev.index)  # host -> device
+            h2d += 3 * 4 * g.n
+            lib.sa_run(ins, chains, steps, seed=RUN_SEED, chain_offset=rank * chains)
+            if world > 1:
+                cdist.global_best(ins, chains)
+            pen, perm, gid = lib.best_get(ins)  # device -> host
+            d2h += 8 + 2 * g.n
+            ins.destroy()
+        return h2d, d2h
+
+    step()
+    torch.cuda.synchronize()
+    if world > 1:
+        torch.distributed.barrier()
+    t = time.perf_counter()
+    for _ in range(k):
+        h2d, d2h = step()
+    torch.cuda.synchronize()
+    dt = time.perf_counter() - t
+    if world > 1:
+        tt = torch.tensor([dt], device=dev, dtype=torch.float64)
+        torch.distributed.all_reduce(tt, op=torch.distributed.ReduceOp.MAX)
+        dt = float(tt.item())
+    evals = _evals_per_step(chains, steps, T0_SAMPLES, len(gens)) * k * world
+    return {"value": evals / dt, "unit": "evals/s", "h2d_bytes_per_step": h2d,
+            "d2h_bytes_per_step": d2h, "steps": k}
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,165 @@
+/*
+ * cdd.h -- C-ABI of libcdd, the B200 (sm_100a) hot path of Awasthi, Lässig, Leuschner & Weise,
+ * "GPGPU-based Parallel Algorithms for Scheduling Against Due Date" (IPDPSW 2016).
+ *
+ * Citations: P:<line> = /root/reference/PAPER.md line (section / equation / algorithm / table).
+ *
+ * The path: many asynchronous SA chains (Alg. 1) or a DPSO swarm (Alg. 2, eq. (3),
+ * P:236-257) whose inner step is the O(n) optimal-timing routine for a fixed job sequence
+ * (CDD: P:94-122; UCDDCP: P:137-166), followed by a reduction to the best sequence.
+ *
+ * Conventions (all entry points):
+ *   - every call returns a cdd_status; nothing throws across the ABI; cdd_last_error() returns a
+ *     thread-local message for the last non-OK status;
+ *   - argument errors are detected synchronously and nothing is launched;
+ *   - "device" pointers are CUDA device pointers on the instance's device (e.g. torch tensors);
+ *     "host" pointers are ordinary host memory; the caller keeps ownership of both;
+ *   - `stream` is a cudaStream_t passed as void* (NULL = legacy default stream); calls marked
+ *     ASYNC only enqueue work on it; CUDA errors surface as CDD_ECUDA at the call that sees them;
+ *   - const pointers are never written; the library frees nothing it did not allocate.
+ * Job sequences are int16 rows: row b holds a permutation of job ids 0..n-1 in positions 0..n-1 of
+ * a row of stride ld >= n elements (ld % 8 == 0 and a 16-byte aligned base enable vector loads).
+ */
+#ifndef CDD_H
+#define CDD_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define CDD_ABI_VERSION 1
+
+#if defined(__GNUC__)
+#define CDD_API __attribute__((visibility("default")))
+#else
+#define CDD_API
+#endif
+
+typedef enum {
+    CDD_OK = 0,
+    CDD_EINVAL = -1, /* bad argument (null pointer, size, problem/instance mismatch)          */
+    CDD_ERANGE = -2, /* instance outside the supported value ranges (see cdd_instance_create)  */
+    CDD_ENOMEM = -3, /* device allocation failed / workspace too small                         */
+    CDD_ECUDA = -4,  /* CUDA runtime error (message in cdd_last_error)                          */
+    CDD_ESTATE = -5, /* no result available yet (best_get before any run)                       */
+    CDD_EDATA = -6   /* a sequence contained a job id outside [0, n) (reported by cdd_check)    */
+} cdd_status;
+
+typedef enum { CDD_PROBLEM_CDD = 0, CDD_PROBLEM_UCDDCP = 1 } cdd_problem;
+
+/* SA neighbourhood: the paper's move (Pert jobs at random positions shuffled by Fisher-Yates,
+ * P:192) or a plain swap of two random positions. */
+typedef enum { CDD_MOVE_PERT_FY = 0, CDD_MOVE_SWAP = 1 } cdd_move;
+
+typedef struct cdd_instance cdd_instance; /* opaque, library-owned, bound to one device */
+
+/* ------------------------------------------------------------------------------------------ */
+/* Instances (problem data)                                                           */
+/* ------------------------------------------------------------------------------------------ */
+/* Copies the host arrays p, alpha, beta (and m, gamma for UCDDCP; both NULL = CDD only), all
+ * indexed by job id, to device `device`.  Checks (CDD_EINVAL): 1 <= n <= 1024, p_i >= 1,
+ * alpha_i, beta_i >= 0, 0 <= m_i <= p_i, gamma_i >= 0, d >= 0.  CDD_ERANGE if the data does
+ * not fit the packed 32-bit job records of this build (sum alpha, sum beta < 2^16;
+ * (sum alpha + sum beta) * sum p < 2^31; field widths for 32 elements per lane <= 32 bits) --
+ * always true for the Biskup-Feldmann ranges p<=20, alpha<=10, beta<=15 at n <= 1000.
+ * Synchronous.  *out receives the instance. */
+CDD_API int cdd_instance_create(int32_t n, const int32_t *p, const int32_t *alpha, const int32_t *beta,
+                        const int32_t *m, const int32_t *gamma, int64_t d, int device,
+                        cdd_instance **out);
+CDD_API int cdd_instance_destroy(cdd_instance *inst);
+/* n, d, sum of p, and flags (bit0: UCDDCP data present, bit1: d >= sum p). Any out may be NULL. */
+CDD_API int cdd_instance_query(const cdd_instance *inst, int32_t *n, int64_t *d, int64_t *sum_p,
+                       int32_t *flags);
+
+/* ------------------------------------------------------------------------------------------ */
+/* Batched sequence evaluation: layer (ii) of the two-layered approach               */
+/* ------------------------------------------------------------------------------------------ */
+/* ASYNC.  out[b] (device int64) = optimal eq. (1) penalty of sequence row b for the CDD with the
+ * instance's d (restrictive or not) -- the value the linear algorithm of P:94-122 finds.
+ * perms: device int16 [batch][ld].  A job id outside [0,n) is treated as an empty job and raises
+ * the instance's data-error flag (see cdd_check); duplicates are not detected. */
+CDD_API int cdd_eval_batch(cdd_instance *inst, const int16_t *perms, int64_t ld, int64_t batch,
+                   int64_t *out, void *stream);
+/* ASYNC.  As above for the UCDDCP objective eq. (2).  CDD_EINVAL if the instance has
+ * no m/gamma or d < sum p (the paper defines the algorithm for the unrestricted case). */
+CDD_API int ucddcp_eval_batch(cdd_instance *inst, const int16_t *perms, int64_t ld, int64_t batch,
+                      int64_t *out, void *stream);
+/* SYNCHRONOUS end-to-end variant with HOST buffers: copies perms_host (int16 [batch][ld]) to the
+ * device in chunks, evaluates, copies the penalties to out_host (int64 [batch]), synchronises. */
+CDD_API int cdd_eval_batch_host(cdd_instance *inst, cdd_problem problem, const int16_t *perms_host,
+                        int64_t ld, int64_t batch, int64_t *out_host, void *stream);
+/* Synchronises `stream`; returns CDD_EDATA (and clears the flag) if any evaluated sequence held
+ * a job id outside [0, n) since the last check, else CDD_OK. */
+CDD_API int cdd_check(cdd_instance *inst, void *stream);
+
+/* ------------------------------------------------------------------------------------------ */
+/* Asynchronous parallel SA (Alg. 1)                                                */
+/* ------------------------------------------------------------------------------------------ */
+typedef struct {
+    cdd_problem problem;
+    int64_t chains;        /* chains on this device (one warp each)                            */
+    int64_t steps;         /* Alg. 1 #Iterations (1000 / 5000)                       */
+    double mu;             /* exponential cooling factor (0.88)                          */
+    double T0;             /* > 0: initial temperature; <= 0: T0 = std of t0_samples random    */
+                           /* sequences, computed on the device                          */
+    int64_t t0_samples;    /* 5000 (used when T0 <= 0)                                   */
+    int32_t pert;          /* perturbation size (4); 1 <= pert <= 4                      */
+    cdd_move move;
+    uint64_t seed;         /* Philox key                                                        */
+    uint64_t chain_offset; /* global id of local chain 0 (multi-GPU: rank * chains);            */
+                           /* chain_offset + chains <= 2^32                                     */
+    int64_t *trace;        /* optional device int64 [chains][steps]: (E_new << 1) | accepted    */
+    int64_t *chain_best;   /* optional device int64 [chains]: best penalty of each chain        */
+    int64_t *chain_final;  /* optional device int64 [chains]: final penalty of each chain       */
+    double *T0_out;        /* optional device double [1]: the T0 used                            */
+    const double *T0_in;   /* optional device double [1]: T0 read on the device (e.g. from sa_t0); */
+                           /* overrides T0 / t0_samples when non-NULL                             */
+} sa_params;
+
+/* Bytes of device workspace sa_run needs for these parameters (caller allocates, e.g. torch). */
+CDD_API size_t sa_workspace_size(const cdd_instance *inst, const sa_params *params);
+/* ASYNC.  Runs params->chains independent chains to completion in one persistent kernel, then
+ * reduces min (best penalty, global chain id) into the instance's best buffers. */
+CDD_API int sa_run(cdd_instance *inst, const sa_params *params, void *workspace, size_t workspace_bytes,
+           void *stream);
+/* ASYNC.  Only the T0 rule: *T0_dev = population std of the penalties of `samples`
+ * Philox-random sequences.  Workspace: sa_workspace_size() of an sa_params with T0 <= 0. */
+CDD_API int sa_t0(cdd_instance *inst, cdd_problem problem, uint64_t seed, int64_t samples, double *T0_dev,
+          void *workspace, size_t workspace_bytes, void *stream);
+
+/* ------------------------------------------------------------------------------------------ */
+/* Discrete PSO (Alg. 2, eq. (3))                                                   */
+/* ------------------------------------------------------------------------------------------ */
+typedef struct {
+    cdd_problem problem;
+    int64_t particles;        /* swarm size on this device                                     */
+    int64_t iters;            /* Alg. 2 #Iterations                                            */
+    double w, c1, c2;         /* probabilities of F1 / F2 / F3 in eq. (3) (silent in the paper)  */
+    uint64_t seed;
+    int64_t *gbest_trace;     /* optional device int64 [iters]: swarm best value at line 5      */
+} dpso_params;
+CDD_API size_t dpso_workspace_size(const cdd_instance *inst, const dpso_params *params);
+/* ASYNC.  Single-device swarm; the final swarm best goes to the instance's best buffers. */
+CDD_API int dpso_run(cdd_instance *inst, const dpso_params *params, void *workspace,
+             size_t workspace_bytes, void *stream);
+
+/* ------------------------------------------------------------------------------------------ */
+/* Best result of the last run (SA or DPSO) on this instance                                   */
+/* ------------------------------------------------------------------------------------------ */
+/* Library-owned device buffers: packed int64 key = (penalty << 32) | global id (min = best,
+ * ties to the lowest id) and int16 [n] sequence.  Valid until the next run or destroy.  The
+ * caller may all-reduce the key (MIN) and broadcast the sequence across GPUs in place. */
+CDD_API int best_device_ptrs(cdd_instance *inst, int64_t **packed_dev, int16_t **perm_dev);
+/* SYNCHRONOUS: penalty, sequence (host int16 [n], may be NULL) and global chain/particle id. */
+CDD_API int best_get(cdd_instance *inst, int64_t *penalty, int16_t *perm_host, uint64_t *id, void *stream);
+
+CDD_API const char *cdd_last_error(void);
+CDD_API int cdd_abi_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* CDD_H */

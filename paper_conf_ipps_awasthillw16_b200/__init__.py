@@ -1,0 +1,306 @@
+"""B200-native hot path of Awasthi, Lässig, Leuschner & Weise, "GPGPU-based Parallel Algorithms for
+Scheduling Against Due Date" (IPDPSW 2016): parallel SA chains / a DPSO swarm over the O(n)
+optimal-timing routine for CDD and UCDDCP job sequences.
+
+This module is the thin Python binding of ``libcdd.so`` (C-ABI declared in ``include/cdd.h``):
+argument marshalling only -- every step of the path runs in the CUDA kernels.  PyTorch provides
+device memory (tensors, workspaces), streams and process groups.  There is no CPU fallback: if
+the library is missing, importing this package fails.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+import re
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SO = os.path.join(_HERE, "libcdd.so")
+HEADER = os.path.join(os.path.dirname(_HERE), "include", "cdd.h")
+
+if not os.path.exists(_SO):
+    raise ImportError(
+        f"libcdd.so not found at {_SO}: build it with `python -c 'import __graft_entry__ as g; "
+        f"g.build()'` (there is no CPU fallback)")
+
+_lib = C.CDLL(_SO)
+
+CDD_OK, CDD_EINVAL, CDD_ERANGE, CDD_ENOMEM, CDD_ECUDA, CDD_ESTATE, CDD_EDATA = 0, -1, -2, -3, -4, -5, -6
+PROBLEMS = {"cdd": 0, "ucddcp": 1}
+MOVES = {"pert_fy": 0, "swap": 1}
+
+
+class CddError(RuntimeError):
+    def __init__(self, code, msg):
+        super().__init__(f"libcdd error {code}: {msg}")
+        self.code = code
+
+
+class SaParams(C.Structure):
+    _fields_ = [("problem", C.c_int), ("chains", C.c_int64), ("steps", C.c_int64),
+                ("mu", C.c_double), ("T0", C.c_double), ("t0_samples", C.c_int64),
+                ("pert", C.c_int32), ("move", C.c_int), ("seed", C.c_uint64),
+                ("chain_offset", C.c_uint64), ("trace", C.c_void_p), ("chain_best", C.c_void_p),
+                ("chain_final", C.c_void_p), ("T0_out", C.c_void_p), ("T0_in", C.c_void_p)]
+
+
+class DpsoParams(C.Structure):
+    _fields_ = [("problem", C.c_int), ("particles", C.c_int64), ("iters", C.c_int64),
+                ("w", C.c_double), ("c1", C.c_double), ("c2", C.c_double), ("seed", C.c_uint64),
+                ("gbest_trace", C.c_void_p)]
+
+
+_vp, _i32, _i64, _u64, _sz = C.c_void_p, C.c_int32, C.c_int64, C.c_uint64, C.c_size_t
+_SIGS = {
+    "cdd_instance_create": (C.c_int, [_i32, _vp, _vp, _vp, _vp, _vp, _i64, C.c_int, C.POINTER(_vp)]),
+    "cdd_instance_destroy": (C.c_int, [_vp]),
+    "cdd_instance_query": (C.c_int, [_vp, _vp, _vp, _vp, _vp]),
+    "cdd_eval_batch": (C.c_int, [_vp, _vp, _i64, _i64, _vp, _vp]),
+    "ucddcp_eval_batch": (C.c_int, [_vp, _vp, _i64, _i64, _vp, _vp]),
+    "cdd_eval_batch_host": (C.c_int, [_vp, C.c_int, _vp, _i64, _i64, _vp, _vp]),
+    "cdd_check": (C.c_int, [_vp, _vp]),
+    "sa_workspace_size": (_sz, [_vp, C.POINTER(SaParams)]),
+    "sa_run": (C.c_int, [_vp, C.POINTER(SaParams), _vp, _sz, _vp]),
+    "sa_t0": (C.c_int, [_vp, C.c_int, _u64, _i64, _vp, _vp, _sz, _vp]),
+    "dpso_workspace_size": (_sz, [_vp, C.POINTER(DpsoParams)]),
+    "dpso_run": (C.c_int, [_vp, C.POINTER(DpsoParams), _vp, _sz, _vp]),
+    "best_device_ptrs": (C.c_int, [_vp, _vp, _vp]),
+    "best_get": (C.c_int, [_vp, _vp, _vp, _vp, _vp]),
+    "cdd_last_error": (C.c_char_p, []),
+    "cdd_abi_version": (C.c_int, []),
+}
+for _name, (_res, _args) in _SIGS.items():
+    _f = getattr(_lib, _name)
+    _f.restype = _res
+    _f.argtypes = _args
+
+
+def header_functions() -> list[str]:
+    """Function names declared in include/cdd.h."""
+    txt = open(HEADER).read()
+    return sorted(set(re.findall(r"^\s*(?:CDD_API\s+)?(?:const\s+)?[a-z_0-9]+\s*\*?\s*([a-z_0-9]+)\s*\(", txt, re.M)))
+
+
+def _check(rc):
+    if rc != CDD_OK:
+        raise CddError(rc, _lib.cdd_last_error().decode())
+
+
+def _stream(stream):
+    if stream is None:
+        import torch
+
+        return torch.cuda.current_stream().cuda_stream
+    return getattr(stream, "cuda_stream", stream)
+
+
+def _dptr(t):
+    return None if t is None else t.data_ptr()
+
+
+def _i32arr(x):
+    return None if x is None else np.ascontiguousarray(x, dtype=np.int32)
+
+
+class Instance:
+    """A problem instance resident on one GPU (wraps ``cdd_instance*``)."""
+
+    def __init__(self, P, alpha, beta, d, M=None, gamma=None, device=0):
+        P, alpha, beta, M, gamma = map(_i32arr, (P, alpha, beta, M, gamma))
+        self.n = int(P.shape[0])
+        self.d = int(d)
+        self.device = int(device)
+        h = _vp()
+        _check(_lib.cdd_instance_create(self.n, P.ctypes.data, alpha.ctypes.data, beta.ctypes.data,
+                                        None if M is None else M.ctypes.data,
+                                        None if gamma is None else gamma.ctypes.data,
+                                        self.d, self.device, C.byref(h)))
+        self._h = h
+        self.sum_p = int(P.sum())
+
+    @classmethod
+    def from_gen(cls, inst, device=0):
+        return cls(inst.P, inst.alpha, inst.beta, inst.d, inst.M, inst.gamma, device)
+
+    @property
+    def handle(self):
+        if self._h is None:
+            raise CddError(CDD_EINVAL, "instance destroyed")
+        return self._h
+
+    def destroy(self):
+        if getattr(self, "_h", None) is not None:
+            _lib.cdd_instance_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.destroy()
+        except Exception:
+            pass
+
+
+def cdd_instance_create(P, alpha, beta, d, M=None, gamma=None, device=0) -> Instance:
+    return Instance(P, alpha, beta, d, M, gamma, device)
+
+
+def cdd_instance_destroy(inst: Instance) -> None:
+    inst.destroy()
+
+
+def _eval(fn, inst, perms, out, stream):
+    import torch
+
+    assert perms.dtype == torch.int16 and perms.dim() == 2 and perms.is_cuda
+    assert perms.stride(1) == 1
+    B, ld = perms.shape[0], perms.stride(0)
+    if out is None:
+        out = torch.empty(B, dtype=torch.int64, device=perms.device)
+    _check(fn(inst.handle, perms.data_ptr(), ld, B, out.data_ptr(), _stream(stream)))
+    return out
+
+
+def cdd_eval_batch(inst: Instance, perms, out=None, stream=None):
+    """out[b] = optimal CDD penalty of sequence perms[b, :n] (device int16 [B, ld])."""
+    return _eval(_lib.cdd_eval_batch, inst, perms, out, stream)
+
+
+def ucddcp_eval_batch(inst: Instance, perms, out=None, stream=None):
+    """out[b] = optimal UCDDCP penalty of sequence perms[b, :n]."""
+    return _eval(_lib.ucddcp_eval_batch, inst, perms, out, stream)
+
+
+def cdd_eval_batch_host(inst: Instance, perms: np.ndarray, problem="cdd", out=None, stream=None):
+    """End-to-end evaluation of HOST sequences (int16 [B, ld]) into a host int64 array."""
+    perms = np.ascontiguousarray(perms, dtype=np.int16) if isinstance(perms, np.ndarray) else perms
+    if isinstance(perms, np.ndarray):
+        B, ld = perms.shape
+        pptr = perms.ctypes.data
+    else:  # pinned torch CPU tensor
+        B, ld = perms.shape
+        pptr = perms.data_ptr()
+    if out is None:
+        out = np.empty(B, dtype=np.int64)
+    optr = out.ctypes.data if isinstance(out, np.ndarray) else out.data_ptr()
+    _check(_lib.cdd_eval_batch_host(inst.handle, PROBLEMS[problem], pptr, ld, B, optr,
+                                    _stream(stream)))
+    return out
+
+
+def cdd_check(inst: Instance, stream=None) -> None:
+    _check(_lib.cdd_check(inst.handle, _stream(stream)))
+
+
+def _sa_params(problem, chains, steps, mu, T0, t0_samples, pert, move, seed, chain_offset,
+               trace=None, chain_best=None, chain_final=None, T0_out=None, T0_in=None):
+    return SaParams(PROBLEMS[problem], int(chains), int(steps), float(mu), float(T0),
+                    int(t0_samples), int(pert), MOVES[move], int(seed) & (2**64 - 1),
+                    int(chain_offset), _dptr(trace), _dptr(chain_best), _dptr(chain_final),
+                    _dptr(T0_out), _dptr(T0_in))
+
+
+def sa_workspace_size(inst: Instance, **kw) -> int:
+    p = _sa_params(**kw)
+    return int(_lib.sa_workspace_size(inst.handle, C.byref(p)))
+
+
+def sa_run(inst: Instance, chains: int, steps: int, problem="cdd", mu=0.88, T0=0.0,
+           t0_samples=5000, pert=4, move="pert_fy", seed=0, chain_offset=0, trace=False,
+           chain_best=False, chain_final=False, stream=None, workspace=None, T0_dev=None):
+    """Asynchronous parallel SA (Alg. 1): `chains` independent chains of `steps` iterations,
+    reduced to the best (penalty, chain) into the instance's best buffers.  Returns the optional
+    per-chain device tensors (and the T0 used) without synchronising."""
+    import torch
+
+    dev = torch.device("cuda", inst.device)
+    res = {"T0": torch.empty(1, dtype=torch.float64, device=dev)}
+    if trace:
+        res["trace"] = torch.empty((chains, steps), dtype=torch.int64, device=dev)
+    if chain_best:
+        res["chain_best"] = torch.empty(chains, dtype=torch.int64, device=dev)
+    if chain_final:
+        res["chain_final"] = torch.empty(chains, dtype=torch.int64, device=dev)
+    p = _sa_params(problem, chains, steps, mu, T0, t0_samples, pert, move, seed, chain_offset,
+                   res.get("trace"), res.get("chain_best"), res.get("chain_final"), res["T0"],
+                   T0_dev)
+    need = int(_lib.sa_workspace_size(inst.handle, C.byref(p)))
+    if need == 0:
+        _check(_lib.sa_run(inst.handle, C.byref(p), None, 0, None))  # raises with the reason
+    if workspace is None or workspace.numel() < need:
+        workspace = torch.empty(need, dtype=torch.uint8, device=dev)
+    res["workspace"] = workspace
+    _check(_lib.sa_run(inst.handle, C.byref(p), workspace.data_ptr(), need, _stream(stream)))
+    return res
+
+
+def sa_t0(inst: Instance, problem="cdd", seed=0, samples=5000, stream=None):
+    """T0 rule of P:192 on the device: population std of `samples` random sequences."""
+    import torch
+
+    dev = torch.device("cuda", inst.device)
+    p = _sa_params(problem, 1, 0, 0.88, 0.0, samples, 4, "pert_fy", seed, 0)
+    need = int(_lib.sa_workspace_size(inst.handle, C.byref(p)))
+    ws = torch.empty(max(need, 1), dtype=torch.uint8, device=dev)
+    T0 = torch.empty(1, dtype=torch.float64, device=dev)
+    _check(_lib.sa_t0(inst.handle, PROBLEMS[problem], int(seed), int(samples), T0.data_ptr(),
+                      ws.data_ptr(), need, _stream(stream)))
+    return T0
+
+
+def dpso_run(inst: Instance, particles: int, iters: int, problem="cdd", w=0.5, c1=0.5, c2=0.5,
+             seed=0, trace=False, stream=None, workspace=None):
+    """Discrete PSO (Alg. 2, eq. (3)) on one GPU; best into the instance's best buffers."""
+    import torch
+
+    dev = torch.device("cuda", inst.device)
+    res = {}
+    if trace:
+        res["gbest_trace"] = torch.empty(iters, dtype=torch.int64, device=dev)
+    p = DpsoParams(PROBLEMS[problem], int(particles), int(iters), float(w), float(c1), float(c2),
+                   int(seed), _dptr(res.get("gbest_trace")))
+    need = int(_lib.dpso_workspace_size(inst.handle, C.byref(p)))
+    if need == 0:
+        _check(_lib.dpso_run(inst.handle, C.byref(p), None, 0, None))
+    if workspace is None or workspace.numel() < need:
+        workspace = torch.empty(need, dtype=torch.uint8, device=dev)
+    res["workspace"] = workspace
+    _check(_lib.dpso_run(inst.handle, C.byref(p), workspace.data_ptr(), need, _stream(stream)))
+    return res
+
+
+def best_device_ptrs(inst: Instance):
+    key = _vp()
+    perm = _vp()
+    _check(_lib.best_device_ptrs(inst.handle, C.byref(key), C.byref(perm)))
+    return key.value, perm.value
+
+
+class _CudaArray:
+    def __init__(self, ptr, shape, typestr):
+        self.__cuda_array_interface__ = {"shape": shape, "typestr": typestr, "data": (ptr, False),
+                                         "version": 3, "strides": None}
+
+
+def best_device_tensors(inst: Instance):
+    """Torch views (no copy) of the instance's best buffers: packed int64 key [1], int16 [n]."""
+    import torch
+
+    kp, pp = best_device_ptrs(inst)
+    dev = torch.device("cuda", inst.device)
+    key = torch.as_tensor(_CudaArray(kp, (1,), "<i8"), device=dev)
+    perm = torch.as_tensor(_CudaArray(pp, (inst.n,), "<i2"), device=dev)
+    return key, perm
+
+
+def best_get(inst: Instance, stream=None):
+    """(penalty, sequence as np.int16[n], global chain/particle id) -- synchronises."""
+    pen = C.c_int64()
+    gid = C.c_uint64()
+    perm = np.zeros(inst.n, dtype=np.int16)
+    _check(_lib.best_get(inst.handle, C.byref(pen), perm.ctypes.data, C.byref(gid), _stream(stream)))
+    return pen.value, perm, gid.value
+
+
+def abi_version() -> int:
+    return int(_lib.cdd_abi_version())

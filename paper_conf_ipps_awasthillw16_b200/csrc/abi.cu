@@ -1,0 +1,411 @@
+// abi.cu -- the C-ABI of libcdd (include/cdd.h): argument checks, instance management, packed
+// record construction, and the launch of the kernels in eval.cu / sa.cu / dpso.cu.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <climits>
+#include <cmath>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "../../include/cdd.h"
+#include "internal.h"
+
+using cdd::Instance;
+
+struct cdd_instance : Instance {};
+
+namespace {
+
+thread_local std::string g_err;
+
+int fail(int code, const std::string& msg) {
+    g_err = msg;
+    return code;
+}
+
+int cuda_fail(cudaError_t e, const char* where) {
+    g_err = std::string(where) + ": " + cudaGetErrorString(e);
+    return CDD_ECUDA;
+}
+
+struct DeviceGuard {
+    int prev = -1;
+    explicit DeviceGuard(int d) {
+        cudaGetDevice(&prev);
+        if (prev != d) cudaSetDevice(d);
+    }
+    ~DeviceGuard() {
+        int cur = -1;
+        cudaGetDevice(&cur);
+        if (prev >= 0 && cur != prev) cudaSetDevice(prev);
+    }
+};
+
+int bits_for(uint64_t v) {
+    int b = 0;
+    while (v) {
+        ++b;
+        v >>= 1;
+    }
+    return b < 1 ? 1 : b;
+}
+
+uint32_t mask_of(int w) { return w >= 32 ? 0xffffffffu : ((1u << w) - 1u); }
+
+cudaStream_t as_stream(void* s) { return reinterpret_cast<cudaStream_t>(s); }
+
+void free_instance(cdd_instance* I) {
+    if (!I) return;
+    DeviceGuard g(I->device);
+    cudaFree(I->rec_cdd);
+    cudaFree(I->rec_ucd);
+    cudaFree(I->err);
+    cudaFree(I->best_key);
+    cudaFree(I->best_perm);
+    cudaFree(I->stage_perm);
+    cudaFree(I->stage_out);
+    delete I;
+}
+
+}  // namespace
+
+extern "C" {
+
+const char* cdd_last_error(void) { return g_err.c_str(); }
+int cdd_abi_version(void) { return CDD_ABI_VERSION; }
+
+int cdd_instance_create(int32_t n, const int32_t* p, const int32_t* alpha, const int32_t* beta,
+                        const int32_t* m, const int32_t* gamma, int64_t d, int device,
+                        cdd_instance** out) {
+    if (!out) return fail(CDD_EINVAL, "out is NULL");
+    *out = nullptr;
+    if (n < 1 || n > 1024) return fail(CDD_EINVAL, "n must be in [1, 1024]");
+    if (!p || !alpha || !beta) return fail(CDD_EINVAL, "p, alpha, beta must be non-NULL");
+    if ((m == nullptr) != (gamma == nullptr)) return fail(CDD_EINVAL, "m and gamma must both be given or both NULL");
+    if (d < 0) return fail(CDD_EINVAL, "d must be >= 0");
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || device < 0 || device >= ndev)
+        return fail(CDD_EINVAL, "invalid CUDA device");
+    int64_t sp = 0, sa = 0, sb = 0;
+    int32_t pmax = 0, amax = 0, bmax = 0, mmax = 0, xmax = 0, gmax = 0;
+    for (int i = 0; i < n; ++i) {
+        if (p[i] < 1) return fail(CDD_EINVAL, "p_i must be >= 1");
+        if (alpha[i] < 0 || beta[i] < 0) return fail(CDD_EINVAL, "alpha_i, beta_i must be >= 0");
+        sp += p[i];
+        sa += alpha[i];
+        sb += beta[i];
+        pmax = std::max(pmax, p[i]);
+        amax = std::max(amax, alpha[i]);
+        bmax = std::max(bmax, beta[i]);
+        if (m) {
+            if (m[i] < 0 || m[i] > p[i]) return fail(CDD_EINVAL, "need 0 <= m_i <= p_i");
+            if (gamma[i] < 0) return fail(CDD_EINVAL, "gamma_i must be >= 0");
+            mmax = std::max(mmax, m[i]);
+            xmax = std::max(xmax, p[i] - m[i]);
+            gmax = std::max(gmax, gamma[i]);
+        }
+    }
+    if (sa >= 65536 || sb >= 65536) return fail(CDD_ERANGE, "sum alpha and sum beta must be < 2^16");
+    if ((sa + sb) * sp >= (int64_t)INT32_MAX) return fail(CDD_ERANGE, "(sum alpha + sum beta) * sum p must be < 2^31");
+    // CDD record: p | a << sa | b << sb, fields wide enough for the sum of 32 records
+    const int wp = bits_for(32ull * (uint64_t)pmax), wa = bits_for(32ull * (uint64_t)amax),
+              wb = bits_for(32ull * (uint64_t)bmax);
+    if (wp + wa + wb > 32) return fail(CDD_ERANGE, "p/alpha/beta too large for 32-bit packed records");
+    auto* I = new cdd_instance();
+    I->device = device;
+    I->n = n;
+    I->d = d;
+    I->sum_p = sp;
+    I->d_eff = (int32_t)std::min<int64_t>(d, sp);
+    I->lay_cdd.sa = wp;
+    I->lay_cdd.sb = wp + wa;
+    I->lay_cdd.pmask = mask_of(wp);
+    I->lay_cdd.amask = mask_of(wa);
+    I->lay_cdd.bmask = mask_of(32 - wp - wa);
+    std::vector<uint32_t> rc(n), ru;
+    for (int i = 0; i < n; ++i)
+        rc[i] = (uint32_t)p[i] | ((uint32_t)alpha[i] << I->lay_cdd.sa) | ((uint32_t)beta[i] << I->lay_cdd.sb);
+    if (m) {
+        const int ua = bits_for(32ull * (uint64_t)amax), ub = bits_for(32ull * (uint64_t)bmax);
+        const int um = bits_for((uint64_t)mmax), ux = bits_for((uint64_t)xmax), ug = bits_for((uint64_t)gmax);
+        if (ua + ub + um + ux + ug <= 32) {
+            I->has_ucd = true;
+            auto& L = I->lay_ucd;
+            L.amask = mask_of(ua);
+            L.sb = ua;
+            L.bmask = mask_of(ub);
+            L.sm = ua + ub;
+            L.mmask = mask_of(um);
+            L.sx = L.sm + um;
+            L.xmask = mask_of(ux);
+            L.sg = L.sx + ux;
+            ru.resize(n);
+            for (int i = 0; i < n; ++i)
+                ru[i] = (uint32_t)alpha[i] | ((uint32_t)beta[i] << L.sb) | ((uint32_t)m[i] << L.sm) |
+                        ((uint32_t)(p[i] - m[i]) << L.sx) | ((uint32_t)gamma[i] << L.sg);
+        } else {
+            delete I;
+            return fail(CDD_ERANGE, "UCDDCP data too large for 32-bit packed records");
+        }
+    }
+    DeviceGuard g(device);
+    cudaError_t e = cudaSuccess;
+    auto chk = [&](cudaError_t x) {
+        if (e == cudaSuccess) e = x;
+    };
+    chk(cudaMalloc(&I->rec_cdd, sizeof(uint32_t) * n));
+    if (I->has_ucd) chk(cudaMalloc(&I->rec_ucd, sizeof(uint32_t) * n));
+    chk(cudaMalloc(&I->err, sizeof(int)));
+    chk(cudaMalloc(&I->best_key, sizeof(unsigned long long)));
+    chk(cudaMalloc(&I->best_perm, sizeof(int16_t) * n));
+    if (e == cudaSuccess) {
+        chk(cudaMemcpy(I->rec_cdd, rc.data(), sizeof(uint32_t) * n, cudaMemcpyHostToDevice));
+        if (I->has_ucd) chk(cudaMemcpy(I->rec_ucd, ru.data(), sizeof(uint32_t) * n, cudaMemcpyHostToDevice));
+        chk(cudaMemset(I->err, 0, sizeof(int)));
+        chk(cudaMemset(I->best_key, 0xff, sizeof(unsigned long long)));
+        chk(cudaMemset(I->best_perm, 0, sizeof(int16_t) * n));
+    }
+    if (e != cudaSuccess) {
+        free_instance(I);
+        return cuda_fail(e, "cdd_instance_create");
+    }
+    *out = I;
+    return CDD_OK;
+}
+
+int cdd_instance_destroy(cdd_instance* inst) {
+    if (!inst) return fail(CDD_EINVAL, "instance is NULL");
+    free_instance(inst);
+    return CDD_OK;
+}
+
+int cdd_instance_query(const cdd_instance* I, int32_t* n, int64_t* d, int64_t* sum_p, int32_t* flags) {
+    if (!I) return fail(CDD_EINVAL, "instance is NULL");
+    if (n) *n = I->n;
+    if (d) *d = I->d;
+    if (sum_p) *sum_p = I->sum_p;
+    if (flags) *flags = (I->has_ucd ? 1 : 0) | (I->d >= I->sum_p ? 2 : 0);
+    return CDD_OK;
+}
+
+static int check_batch_args(const cdd_instance* I, const int16_t* perms, int64_t ld, int64_t batch,
+                            const int64_t* out) {
+    if (!I) return fail(CDD_EINVAL, "instance is NULL");
+    if (batch < 0) return fail(CDD_EINVAL, "batch must be >= 0");
+    if (batch > 0 && (!perms || !out)) return fail(CDD_EINVAL, "perms/out must be non-NULL");
+    if (ld < I->n) return fail(CDD_EINVAL, "ld must be >= n");
+    return CDD_OK;
+}
+
+static int eval_common(cdd_instance* I, bool ucd, const int16_t* perms, int64_t ld, int64_t batch,
+                       int64_t* out, void* stream) {
+    int rc = check_batch_args(I, perms, ld, batch, out);
+    if (rc != CDD_OK) return rc;
+    if (ucd && !I->has_ucd) return fail(CDD_EINVAL, "instance has no m/gamma (UCDDCP data)");
+    if (ucd && I->d < I->sum_p) return fail(CDD_EINVAL, "UCDDCP needs d >= sum p (unrestricted case, P:126)");
+    DeviceGuard g(I->device);
+    cudaError_t e = cdd::launch_eval_batch(*I, ucd, perms, ld, batch, out, as_stream(stream));
+    return e == cudaSuccess ? CDD_OK : cuda_fail(e, ucd ? "ucddcp_eval_batch" : "cdd_eval_batch");
+}
+
+int cdd_eval_batch(cdd_instance* I, const int16_t* perms, int64_t ld, int64_t batch, int64_t* out,
+                   void* stream) {
+    return eval_common(I, false, perms, ld, batch, out, stream);
+}
+
+int ucddcp_eval_batch(cdd_instance* I, const int16_t* perms, int64_t ld, int64_t batch, int64_t* out,
+                      void* stream) {
+    return eval_common(I, true, perms, ld, batch, out, stream);
+}
+
+int cdd_eval_batch_host(cdd_instance* I, cdd_problem problem, const int16_t* perms_host, int64_t ld,
+                        int64_t batch, int64_t* out_host, void* stream) {
+    int rc = check_batch_args(I, perms_host, ld, batch, out_host);
+    if (rc != CDD_OK) return rc;
+    if (problem != CDD_PROBLEM_CDD && problem != CDD_PROBLEM_UCDDCP) return fail(CDD_EINVAL, "bad problem");
+    const bool ucd = problem == CDD_PROBLEM_UCDDCP;
+    if (ucd && (!I->has_ucd || I->d < I->sum_p)) return fail(CDD_EINVAL, "instance not usable for UCDDCP");
+    DeviceGuard g(I->device);
+    cudaStream_t s = as_stream(stream);
+    const int64_t chunk = std::max<int64_t>(1, std::min<int64_t>(batch, (int64_t)(256ll << 20) / (ld * 2)));
+    if (I->stage_rows < (size_t)chunk * ld) {
+        cudaFree(I->stage_perm);
+        cudaFree(I->stage_out);
+        I->stage_perm = nullptr;
+        I->stage_out = nullptr;
+        I->stage_rows = 0;
+        cudaError_t e = cudaMalloc(&I->stage_perm, sizeof(int16_t) * (size_t)chunk * ld);
+        if (e == cudaSuccess) e = cudaMalloc(&I->stage_out, sizeof(int64_t) * (size_t)chunk);
+        if (e != cudaSuccess) return cuda_fail(e, "cdd_eval_batch_host staging");
+        I->stage_rows = (size_t)chunk * ld;
+    }
+    for (int64_t a = 0; a < batch; a += chunk) {
+        const int64_t rows = std::min(chunk, batch - a);
+        cudaError_t e = cudaMemcpyAsync(I->stage_perm, perms_host + a * ld, sizeof(int16_t) * rows * ld,
+                                        cudaMemcpyHostToDevice, s);
+        if (e == cudaSuccess) e = cdd::launch_eval_batch(*I, ucd, I->stage_perm, ld, rows, I->stage_out, s);
+        if (e == cudaSuccess)
+            e = cudaMemcpyAsync(out_host + a, I->stage_out, sizeof(int64_t) * rows, cudaMemcpyDeviceToHost, s);
+        if (e != cudaSuccess) return cuda_fail(e, "cdd_eval_batch_host");
+    }
+    cudaError_t e = cudaStreamSynchronize(s);
+    return e == cudaSuccess ? CDD_OK : cuda_fail(e, "cdd_eval_batch_host sync");
+}
+
+int cdd_check(cdd_instance* I, void* stream) {
+    if (!I) return fail(CDD_EINVAL, "instance is NULL");
+    DeviceGuard g(I->device);
+    cudaStream_t s = as_stream(stream);
+    int flag = 0;
+    cudaError_t e = cudaMemcpyAsync(&flag, I->err, sizeof(int), cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+    if (e != cudaSuccess) return cuda_fail(e, "cdd_check");
+    if (flag) {
+        cudaMemsetAsync(I->err, 0, sizeof(int), s);
+        cudaStreamSynchronize(s);
+        return fail(CDD_EDATA, "a sequence contained a job id outside [0, n)");
+    }
+    return CDD_OK;
+}
+
+static int sa_validate(const cdd_instance* I, const sa_params* p, cdd::SaLaunch* L) {
+    if (!I || !p) return fail(CDD_EINVAL, "instance/params is NULL");
+    if (p->problem != CDD_PROBLEM_CDD && p->problem != CDD_PROBLEM_UCDDCP) return fail(CDD_EINVAL, "bad problem");
+    const bool ucd = p->problem == CDD_PROBLEM_UCDDCP;
+    if (ucd && (!I->has_ucd || I->d < I->sum_p)) return fail(CDD_EINVAL, "instance not usable for UCDDCP");
+    if (p->chains < 1) return fail(CDD_EINVAL, "chains must be >= 1");
+    if (p->steps < 0 || p->steps >= (int64_t)UINT32_MAX) return fail(CDD_EINVAL, "steps must be in [0, 2^32)");
+    if (p->chain_offset + (uint64_t)p->chains > (1ull << 32)) return fail(CDD_EINVAL, "chain ids must fit 32 bits");
+    if (p->pert < 1 || p->pert > 4) return fail(CDD_EINVAL, "pert must be in [1, 4]");
+    if (p->move != CDD_MOVE_PERT_FY && p->move != CDD_MOVE_SWAP) return fail(CDD_EINVAL, "bad move");
+    if (!std::isfinite(p->mu) || p->mu < 0) return fail(CDD_EINVAL, "mu must be finite and >= 0");
+    if (!(p->T0 > 0) && !p->T0_in && p->t0_samples < 1) return fail(CDD_EINVAL, "T0 <= 0 needs t0_samples >= 1");
+    if (std::isnan(p->T0)) return fail(CDD_EINVAL, "T0 is NaN");
+    L->ucd = ucd;
+    L->chains = p->chains;
+    L->steps = p->steps;
+    L->mu = p->mu;
+    L->T0 = p->T0_in ? 1.0 : p->T0;
+    L->t0_samples = (p->T0 > 0 || p->T0_in) ? 0 : p->t0_samples;
+    L->T0_in = p->T0_in;
+    L->pert = p->pert;
+    L->move = (int32_t)p->move;
+    L->seed = p->seed;
+    L->chain_offset = p->chain_offset;
+    L->trace = p->trace;
+    L->chain_best = p->chain_best;
+    L->chain_final = p->chain_final;
+    L->T0_out = p->T0_out;
+    return CDD_OK;
+}
+
+size_t sa_workspace_size(const cdd_instance* I, const sa_params* p) {
+    cdd::SaLaunch L{};
+    if (sa_validate(I, p, &L) != CDD_OK) return 0;
+    DeviceGuard g(I->device);
+    return cdd::sa_workspace_bytes(*I, L);
+}
+
+int sa_run(cdd_instance* I, const sa_params* p, void* ws, size_t ws_bytes, void* stream) {
+    cdd::SaLaunch L{};
+    int rc = sa_validate(I, p, &L);
+    if (rc != CDD_OK) return rc;
+    DeviceGuard g(I->device);
+    const size_t need = cdd::sa_workspace_bytes(*I, L);
+    if (!ws || ws_bytes < need)
+        return fail(CDD_ENOMEM, "workspace too small: need " + std::to_string(need) + " bytes");
+    cudaError_t e = cdd::launch_sa(*I, L, ws, as_stream(stream));
+    if (e != cudaSuccess) return cuda_fail(e, "sa_run");
+    I->has_best = true;
+    return CDD_OK;
+}
+
+int sa_t0(cdd_instance* I, cdd_problem problem, uint64_t seed, int64_t samples, double* T0_dev,
+          void* ws, size_t ws_bytes, void* stream) {
+    if (!I || !T0_dev) return fail(CDD_EINVAL, "instance/T0_dev is NULL");
+    if (samples < 1) return fail(CDD_EINVAL, "samples must be >= 1");
+    sa_params p{};
+    p.problem = problem;
+    p.chains = 1;
+    p.steps = 0;
+    p.mu = 0.88;
+    p.T0 = 0;
+    p.t0_samples = samples;
+    p.pert = 4;
+    cdd::SaLaunch L{};
+    int rc = sa_validate(I, &p, &L);
+    if (rc != CDD_OK) return rc;
+    DeviceGuard g(I->device);
+    const size_t need = cdd::sa_workspace_bytes(*I, L);
+    if (!ws || ws_bytes < need)
+        return fail(CDD_ENOMEM, "workspace too small: need " + std::to_string(need) + " bytes");
+    cudaError_t e = cdd::launch_t0(*I, L.ucd, seed, samples, T0_dev, ws, as_stream(stream));
+    return e == cudaSuccess ? CDD_OK : cuda_fail(e, "sa_t0");
+}
+
+static int dpso_validate(const cdd_instance* I, const dpso_params* p, cdd::DpsoLaunch* L) {
+    if (!I || !p) return fail(CDD_EINVAL, "instance/params is NULL");
+    if (p->problem != CDD_PROBLEM_CDD && p->problem != CDD_PROBLEM_UCDDCP) return fail(CDD_EINVAL, "bad problem");
+    const bool ucd = p->problem == CDD_PROBLEM_UCDDCP;
+    if (ucd && (!I->has_ucd || I->d < I->sum_p)) return fail(CDD_EINVAL, "instance not usable for UCDDCP");
+    if (I->n < 2) return fail(CDD_EINVAL, "DPSO needs n >= 2");
+    if (p->particles < 1 || p->particles >= (1ll << 31)) return fail(CDD_EINVAL, "particles must be in [1, 2^31)");
+    if (p->iters < 0 || p->iters >= (int64_t)UINT32_MAX) return fail(CDD_EINVAL, "iters must be in [0, 2^32)");
+    L->ucd = ucd;
+    L->particles = p->particles;
+    L->iters = p->iters;
+    L->w = p->w;
+    L->c1 = p->c1;
+    L->c2 = p->c2;
+    L->seed = p->seed;
+    L->gbest_trace = p->gbest_trace;
+    return CDD_OK;
+}
+
+size_t dpso_workspace_size(const cdd_instance* I, const dpso_params* p) {
+    cdd::DpsoLaunch L{};
+    if (dpso_validate(I, p, &L) != CDD_OK) return 0;
+    return cdd::dpso_workspace_bytes(*I, L);
+}
+
+int dpso_run(cdd_instance* I, const dpso_params* p, void* ws, size_t ws_bytes, void* stream) {
+    cdd::DpsoLaunch L{};
+    int rc = dpso_validate(I, p, &L);
+    if (rc != CDD_OK) return rc;
+    DeviceGuard g(I->device);
+    const size_t need = cdd::dpso_workspace_bytes(*I, L);
+    if (!ws || ws_bytes < need)
+        return fail(CDD_ENOMEM, "workspace too small: need " + std::to_string(need) + " bytes");
+    cudaError_t e = cdd::launch_dpso(*I, L, ws, as_stream(stream));
+    if (e != cudaSuccess) return cuda_fail(e, "dpso_run");
+    I->has_best = true;
+    return CDD_OK;
+}
+
+int best_device_ptrs(cdd_instance* I, int64_t** packed_dev, int16_t** perm_dev) {
+    if (!I) return fail(CDD_EINVAL, "instance is NULL");
+    if (packed_dev) *packed_dev = reinterpret_cast<int64_t*>(I->best_key);
+    if (perm_dev) *perm_dev = I->best_perm;
+    return CDD_OK;
+}
+
+int best_get(cdd_instance* I, int64_t* penalty, int16_t* perm_host, uint64_t* id, void* stream) {
+    if (!I) return fail(CDD_EINVAL, "instance is NULL");
+    if (!I->has_best) return fail(CDD_ESTATE, "no run has completed on this instance");
+    DeviceGuard g(I->device);
+    cudaStream_t s = as_stream(stream);
+    unsigned long long key = 0;
+    cudaError_t e = cudaMemcpyAsync(&key, I->best_key, sizeof key, cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess && perm_host)
+        e = cudaMemcpyAsync(perm_host, I->best_perm, sizeof(int16_t) * I->n, cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+    if (e != cudaSuccess) return cuda_fail(e, "best_get");
+    if (key == ULLONG_MAX) return fail(CDD_ESTATE, "no result");
+    if (penalty) *penalty = (int64_t)(key >> 32);
+    if (id) *id = key & 0xffffffffull;
+    return CDD_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,77 @@
+// internal.h -- host/device shared declarations of libcdd (not part of the public ABI).
+#pragma once
+#include <cuda_runtime.h>
+
+#include <cstddef>
+#include <cstdint>
+
+namespace cdd {
+
+// Packed 32-bit job record.  CDD: p | a << sa | b << sb (b is the top field).  UCDDCP:
+// a | b << sb | M << sm | X << sx | gamma << sg (gamma top).  Field widths are sized so that
+// the sum of 32 records (one lane's chunk) never carries out of the p, a, b fields, which lets a
+// single integer add form the prefix sums of all three at once.
+struct RecLayout {
+    int32_t sa, sb, sm, sx, sg;
+    uint32_t pmask, amask, bmask, mmask, xmask;
+};
+
+constexpr uint32_t kTagSaInit = 0x11u, kTagSa = 0x12u, kTagT0 = 0x13u, kTagDpsoInit = 0x21u,
+                   kTagDpso = 0x22u;
+
+struct Instance {
+    int device = 0;
+    int32_t n = 0;
+    int64_t d = 0;
+    int64_t sum_p = 0;
+    int32_t d_eff = 0;  // min(d, sum p): CDD penalties do not depend on d beyond sum p
+    bool has_ucd = false;
+    RecLayout lay_cdd{}, lay_ucd{};
+    uint32_t* rec_cdd = nullptr;  // device [n] records by job id
+    uint32_t* rec_ucd = nullptr;
+    int* err = nullptr;                    // device data-error flag
+    unsigned long long* best_key = nullptr;  // device packed (penalty << 32 | id)
+    int16_t* best_perm = nullptr;          // device [n]
+    bool has_best = false;
+    // host e2e staging
+    int16_t* stage_perm = nullptr;
+    int64_t* stage_out = nullptr;
+    size_t stage_rows = 0;
+};
+
+// ---- launchers (eval.cu) ----
+cudaError_t launch_eval_batch(const Instance& I, bool ucd, const int16_t* perms, int64_t ld,
+                              int64_t batch, int64_t* out, cudaStream_t s);
+
+// ---- launchers (sa.cu) ----
+struct SaLaunch {
+    bool ucd;
+    int64_t chains, steps;
+    double mu;
+    double T0;  // <= 0: computed into workspace
+    int64_t t0_samples;
+    int32_t pert, move;
+    uint64_t seed, chain_offset;
+    int64_t *trace, *chain_best, *chain_final;
+    double* T0_out;
+    const double* T0_in;
+};
+size_t sa_workspace_bytes(const Instance& I, const SaLaunch& p);
+cudaError_t launch_t0(const Instance& I, bool ucd, uint64_t seed, int64_t samples, double* T0_dev,
+                      void* ws, cudaStream_t s);
+cudaError_t launch_sa(Instance& I, const SaLaunch& p, void* ws, cudaStream_t s);
+
+// ---- launchers (dpso.cu) ----
+struct DpsoLaunch {
+    bool ucd;
+    int64_t particles, iters;
+    double w, c1, c2;
+    uint64_t seed;
+    int64_t* gbest_trace;
+};
+size_t dpso_workspace_bytes(const Instance& I, const DpsoLaunch& p);
+cudaError_t launch_dpso(Instance& I, const DpsoLaunch& p, void* ws, cudaStream_t s);
+
+int sa_e_for_n(int n);  // elements per lane of the warp-per-chain kernels
+
+}  // namespace cdd

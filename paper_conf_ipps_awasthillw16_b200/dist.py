@@ -1,0 +1,37 @@
+"""Multi-GPU reduction of the best sequence (one process per GPU, torch.distributed).
+
+Asynchronous SA shards naturally: rank r runs global chain ids [r*C, (r+1)*C) with identical
+per-chain Philox streams, so the result does not depend on the number of GPUs.  The
+only exchange is the final reduction of P:226-228 lifted across GPUs: a MIN all-reduce of the packed
+int64 key (penalty << 32 | global chain id) in place on the library's device buffer, then a
+broadcast of the winner's int16 sequence (as uint8: NCCL has no int16) from the owning rank.
+"""
+from __future__ import annotations
+
+import torch
+import torch.distributed as dist
+
+from . import best_device_tensors
+
+
+def owner_rank(key: int, ids_per_rank: int) -> int:
+    """Rank that owns the global id packed in `key` (ids are rank-contiguous)."""
+    return int(key & 0xFFFFFFFF) // int(ids_per_rank)
+
+
+def reduce_best(key: torch.Tensor, perm: torch.Tensor, ids_per_rank: int, group=None) -> int:
+    """In place: key <- MIN over ranks; perm <- the winner's perm.  Returns the winner's rank.
+
+    `key` is an int64 [1] tensor, `perm` an int16 [n] tensor (device tensors with NCCL, CPU tensors
+    with gloo).  One all-reduce and one broadcast; the broadcast source is known to every rank
+    from the reduced key, so no extra round trip is needed."""
+    dist.all_reduce(key, op=dist.ReduceOp.MIN, group=group)
+    src = owner_rank(int(key.item()), ids_per_rank)
+    dist.broadcast(perm.view(torch.uint8), src=src, group=group)
+    return src
+
+
+def global_best(inst, ids_per_rank: int, group=None) -> int:
+    """Reduce the instance's device-resident best (after sa_run / dpso_run) across all ranks."""
+    key, perm = best_device_tensors(inst)
+    return reduce_best(key, perm, ids_per_rank, group)

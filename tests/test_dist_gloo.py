@@ -1,0 +1,76 @@
+"""World-size-2 CPU (gloo) test of the cross-GPU reduction logic (SURVEY T10 sharding invariance).
+
+Each rank runs its shard of SA chains (global ids rank*C .. rank*C+C-1) with the oracle, packs its
+local best as (penalty << 32 | global chain id), and calls the same reduce_best() the GPU path uses
+over NCCL.  The reduced result must equal one run over all 2C chains."""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _worker(rank, world, port, C, q):
+    import sys
+
+    sys.path.insert(0, ROOT)
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    import gen
+    import oracle
+    from paper_conf_ipps_awasthillw16_b200.dist import reduce_best
+
+    inst = gen.cdd_instance(40, 3, 0.4)
+    pr = oracle.Problem.from_instance(inst)
+    T0 = oracle.t0(pr, oracle.CDD, 5, 300)
+    p = oracle.sa_params(chains=C, steps=150, seed=5, chain_offset=rank * C)
+    r = oracle.sa_run(pr, p, T0)
+    key = torch.tensor([(r["E_best"] << 32) | r["g"]], dtype=torch.int64)
+    perm = torch.from_numpy(r["best"].copy())
+    src = reduce_best(key, perm, C)
+    q.put((rank, int(key.item()), perm.numpy().tolist(), src))
+    dist.destroy_process_group()
+
+
+def test_reduce_best_matches_single_run():
+    world, C = 2, 12
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    ps = [ctx.Process(target=_worker, args=(r, world, port, C, q)) for r in range(world)]
+    [p.start() for p in ps]
+    res = [q.get(timeout=120) for _ in range(world)]
+    [p.join(timeout=60) for p in ps]
+    assert all(p.exitcode == 0 for p in ps)
+    import gen
+    import oracle
+
+    inst = gen.cdd_instance(40, 3, 0.4)
+    pr = oracle.Problem.from_instance(inst)
+    T0 = oracle.t0(pr, oracle.CDD, 5, 300)
+    full = oracle.sa_run(pr, oracle.sa_params(chains=world * C, steps=150, seed=5), T0)
+    for rank, key, perm, src in res:
+        assert key >> 32 == full["E_best"] and key & 0xFFFFFFFF == full["g"]
+        assert perm == full["best"].tolist()
+        assert src == full["g"] // C
+
+
+def test_owner_rank():
+    from paper_conf_ipps_awasthillw16_b200.dist import owner_rank
+
+    assert owner_rank((123 << 32) | 70000, 65536) == 1
+    assert owner_rank((5 << 32) | 0, 65536) == 0

@@ -1,0 +1,178 @@
+"""GPU parity: batched evaluation kernels vs the oracle, element by element (bit-exact int64)."""
+import json
+import os
+
+import numpy as np
+import pytest
+
+import gen
+import oracle
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def lib():
+    import torch
+
+    assert torch.cuda.is_available()
+    import paper_conf_ipps_awasthillw16_b200 as m
+
+    return m
+
+
+def _dev(x):
+    import torch
+
+    return torch.from_numpy(np.ascontiguousarray(x)).cuda()
+
+
+def _gpu_eval(lib, inst, perms, problem="cdd", d=None):
+    ins = lib.Instance(inst.P, inst.alpha, inst.beta, inst.d if d is None else d, inst.M, inst.gamma)
+    fn = lib.cdd_eval_batch if problem == "cdd" else lib.ucddcp_eval_batch
+    out = fn(ins, _dev(perms)).cpu().numpy()
+    lib.cdd_check(ins)
+    ins.destroy()
+    return out
+
+
+def _oracle(inst, perms, problem="cdd", d=None):
+    pr = oracle.Problem.from_instance(inst, d=d)
+    return oracle.eval_batch_threaded(pr, perms, oracle.CDD if problem == "cdd" else oracle.UCDDCP)
+
+
+def test_table1(lib):
+    t = gen.table1()
+    perms = gen.random_perms(1, 5, 0)
+    perms[0, :5] = np.arange(5)
+    assert _gpu_eval(lib, t, perms)[0] == 81
+    assert _gpu_eval(lib, t, perms, "ucddcp", d=22)[0] == 77
+
+
+def test_config1_all_10_factorial(lib):
+    # BASELINE config 1: CDD n=10, h=0.4, seed 1 -- every one of the 10! sequences
+    gold = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "config1.json")))
+    inst = gen.cdd_instance(10, 1, 0.4)
+    perms = gen.all_perms(10)
+    z = _gpu_eval(lib, inst, perms)
+    ref = _oracle(inst, perms)
+    assert np.array_equal(z, ref)
+    assert int(z.min()) == gold["optimum"] and int(z.sum()) == gold["z_sum_over_all"]
+
+
+@pytest.mark.parametrize("n", [1, 2, 3, 5, 7, 8, 9, 15, 16, 17, 31, 32, 33, 63, 64, 65, 100, 127,
+                               128, 129, 200, 255, 256, 257, 333, 500, 511, 512, 513, 777, 999,
+                               1000, 1023, 1024])
+def test_random_instances_all_templates(lib, n):
+    rng = np.random.default_rng(n)
+    for h in (0.0, 0.2, 0.4, 0.6, 0.8, 1.0, 1.7):
+        inst = gen.cdd_instance(n, 1 + n % 7, 0.2)
+        d = int(h * inst.sum_p)
+        B = 700 if n <= 256 else 150
+        perms = gen.random_perms(B, n, int(rng.integers(1 << 30)))
+        assert np.array_equal(_gpu_eval(lib, inst, perms, d=d), _oracle(inst, perms, d=d)), (n, h)
+
+
+@pytest.mark.parametrize("n", [1, 4, 10, 17, 50, 100, 129, 200, 300, 500, 640, 1000, 1024])
+def test_ucddcp_random(lib, n):
+    inst = gen.ucddcp_instance(n, 2 + n % 5)
+    B = 600 if n <= 256 else 120
+    perms = gen.random_perms(B, n, 77 + n)
+    for extra in (0, 13):
+        d = inst.sum_p + extra
+        assert np.array_equal(_gpu_eval(lib, inst, perms, "ucddcp", d=d),
+                              _oracle(inst, perms, "ucddcp", d=d)), (n, extra)
+
+
+def test_small_value_instances_and_zero_weights(lib):
+    # tiny values, zero penalties, restrictive and unrestricted due dates
+    for c in range(300):
+        n = 1 + c % 40
+        inst = gen.random_small(n, 9000 + c, pmax=7, wmax=4, zero_weights=(c % 3 == 0))
+        perms = gen.random_perms(64, n, c)
+        assert np.array_equal(_gpu_eval(lib, inst, perms), _oracle(inst, perms)), c
+        if c % 2 == 0:
+            d = inst.sum_p + c % 5
+            assert np.array_equal(_gpu_eval(lib, inst, perms, "ucddcp", d=d),
+                                  _oracle(inst, perms, "ucddcp", d=d)), c
+
+
+def test_config2_shape_n100_all_h(lib):
+    # BASELINE config 2 shape: n=100, h in {0.2,...,0.8}, 10 instances each (20k sequences each)
+    perms = gen.random_perms(20000, 100, 2024)
+    for k in range(1, 11):
+        for h in gen.H_VALUES:
+            inst = gen.cdd_instance(100, k, h)
+            assert np.array_equal(_gpu_eval(lib, inst, perms), _oracle(inst, perms)), (k, h)
+
+
+def test_unaligned_and_odd_stride(lib):
+    import torch
+
+    inst = gen.cdd_instance(100, 3, 0.4)
+    perms = gen.random_perms(999, 100, 5, ld=103)  # ld % 8 != 0 -> scalar loads
+    ref = _oracle(inst, perms)
+    ins = lib.Instance.from_gen(inst)
+    assert np.array_equal(lib.cdd_eval_batch(ins, _dev(perms)).cpu().numpy(), ref)
+    big = torch.zeros((1000, 104), dtype=torch.int16, device="cuda")
+    p8 = gen.random_perms(999, 100, 6, ld=104)
+    big[1:, :] = _dev(p8)
+    view = big[1:]  # 16-B aligned rows; also an unaligned base via a column offset
+    assert np.array_equal(lib.cdd_eval_batch(ins, view).cpu().numpy(), _oracle(inst, p8))
+    flat = torch.zeros(999 * 104 + 1, dtype=torch.int16, device="cuda")
+    un = flat[1:].view(999, 104)
+    un.copy_(_dev(p8))
+    assert np.array_equal(lib.cdd_eval_batch(ins, un).cpu().numpy(), _oracle(inst, p8))
+
+
+def test_invalid_ids_flagged(lib):
+    inst = gen.cdd_instance(50, 1, 0.4)
+    perms = gen.random_perms(10, 50, 1)
+    perms[3, 7] = 50
+    ins = lib.Instance.from_gen(inst)
+    lib.cdd_eval_batch(ins, _dev(perms))
+    with pytest.raises(lib.CddError) as e:
+        lib.cdd_check(ins)
+    assert e.value.code == lib.CDD_EDATA
+    lib.cdd_check(ins)  # flag cleared
+
+
+def test_host_e2e_path(lib):
+    inst = gen.cdd_instance(1000, 1, 0.6)
+    perms = gen.random_perms(3000, 1000, 8)
+    ins = lib.Instance.from_gen(inst)
+    out = lib.cdd_eval_batch_host(ins, perms)
+    assert np.array_equal(out, _oracle(inst, perms))
+
+
+def test_full_size_n1000_bench_launch(lib):
+    # BASELINE metric configuration: n=1000, device-generated sequences (bench launch), sampled
+    import torch
+
+    inst = gen.cdd_instance(1000, 1, 0.4)
+    ins = lib.Instance.from_gen(inst)
+    perms = gen.random_perms_device(1 << 20, 1000, 99)
+    out = lib.cdd_eval_batch(ins, perms)
+    torch.cuda.synchronize()
+    idx = np.random.default_rng(0).choice(perms.shape[0], 4000, replace=False)
+    idx = np.concatenate([idx, [0, perms.shape[0] - 1]])
+    sample = perms[torch.from_numpy(idx).cuda()].cpu().numpy()
+    assert np.array_equal(out.cpu().numpy()[idx], _oracle(inst, sample))
+    # property at full size: every penalty is within [min over sample-free bounds]: Z >= 0 and
+    # Z <= (sum alpha + sum beta) * sum p
+    o = out.cpu().numpy()
+    assert (o >= 0).all() and (o <= (int(inst.alpha.sum()) + int(inst.beta.sum())) * inst.sum_p).all()
+
+
+def test_instance_argument_errors(lib):
+    with pytest.raises(lib.CddError):
+        lib.Instance([0, 1], [1, 1], [1, 1], 3)          # p_i >= 1
+    with pytest.raises(lib.CddError):
+        lib.Instance([1] * 1025, [1] * 1025, [1] * 1025, 3)  # n <= 1024
+    with pytest.raises(lib.CddError) as e:
+        lib.Instance([1000] * 10, [1000] * 10, [1] * 10, 3)
+    assert e.value.code == lib.CDD_ERANGE
+    inst = gen.cdd_instance(20, 1, 0.4)
+    ins = lib.Instance(inst.P, inst.alpha, inst.beta, inst.d)
+    with pytest.raises(lib.CddError):
+        lib.ucddcp_eval_batch(ins, _dev(gen.random_perms(4, 20, 1)))  # no UCDDCP data
