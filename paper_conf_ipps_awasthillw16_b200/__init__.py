@@ -16,7 +16,7 @@ import re
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-_SO = os.path.join(_HERE, "libcdd.so")
+_SO = os.environ.get("CDD_LIB") or os.path.join(_HERE, "libcdd.so")
 HEADER = os.path.join(os.path.dirname(_HERE), "include", "cdd.h")
 
 if not os.path.exists(_SO):

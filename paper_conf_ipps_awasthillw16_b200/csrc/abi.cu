@@ -61,6 +61,11 @@ void free_instance(cdd_instance* I) {
     DeviceGuard g(I->device);
     cudaFree(I->rec_cdd);
     cudaFree(I->rec_ucd);
+    cudaFree(I->tab_ab);
+    cudaFree(I->tab_p);
+    cudaFree(I->tab_m);
+    cudaFree(I->tab_x);
+    cudaFree(I->tab_g);
     cudaFree(I->err);
     cudaFree(I->best_key);
     cudaFree(I->best_perm);
@@ -113,6 +118,10 @@ int cdd_instance_create(int32_t n, const int32_t* p, const int32_t* alpha, const
     const int wp = bits_for(32ull * (uint64_t)pmax), wa = bits_for(32ull * (uint64_t)amax),
               wb = bits_for(32ull * (uint64_t)bmax);
     if (wp + wa + wb > 32) return fail(CDD_ERANGE, "p/alpha/beta too large for 32-bit packed records");
+    // warp-per-chain tables: p, M, P-M in bytes; alpha, beta, gamma in 16-bit halves (lane sums of
+    // alpha and beta over 32 positions must stay below 2^16)
+    if (pmax > 255 || 32 * amax >= 65536 || 32 * bmax >= 65536 || gmax >= 65536 || xmax > 255)
+        return fail(CDD_ERANGE, "need p <= 255, alpha, beta < 2048, gamma < 65536 for the SA tables");
     auto* I = new cdd_instance();
     I->device = device;
     I->n = n;
@@ -160,6 +169,34 @@ int cdd_instance_create(int32_t n, const int32_t* p, const int32_t* alpha, const
     chk(cudaMalloc(&I->err, sizeof(int)));
     chk(cudaMalloc(&I->best_key, sizeof(unsigned long long)));
     chk(cudaMalloc(&I->best_perm, sizeof(int16_t) * n));
+    std::vector<uint32_t> tab(n);
+    std::vector<uint8_t> tp(n), tm(n), tx(n);
+    std::vector<uint16_t> tg(n);
+    for (int i = 0; i < n; ++i) {
+        tab[i] = (uint32_t)alpha[i] | ((uint32_t)beta[i] << 16);
+        tp[i] = (uint8_t)p[i];
+        if (m) {
+            tm[i] = (uint8_t)m[i];
+            tx[i] = (uint8_t)(p[i] - m[i]);
+            tg[i] = (uint16_t)gamma[i];
+        }
+    }
+    chk(cudaMalloc(&I->tab_ab, sizeof(uint32_t) * n));
+    chk(cudaMalloc(&I->tab_p, n));
+    if (I->has_ucd) {
+        chk(cudaMalloc(&I->tab_m, n));
+        chk(cudaMalloc(&I->tab_x, n));
+        chk(cudaMalloc(&I->tab_g, sizeof(uint16_t) * n));
+    }
+    if (e == cudaSuccess) {
+        chk(cudaMemcpy(I->tab_ab, tab.data(), sizeof(uint32_t) * n, cudaMemcpyHostToDevice));
+        chk(cudaMemcpy(I->tab_p, tp.data(), n, cudaMemcpyHostToDevice));
+        if (I->has_ucd) {
+            chk(cudaMemcpy(I->tab_m, tm.data(), n, cudaMemcpyHostToDevice));
+            chk(cudaMemcpy(I->tab_x, tx.data(), n, cudaMemcpyHostToDevice));
+            chk(cudaMemcpy(I->tab_g, tg.data(), sizeof(uint16_t) * n, cudaMemcpyHostToDevice));
+        }
+    }
     if (e == cudaSuccess) {
         chk(cudaMemcpy(I->rec_cdd, rc.data(), sizeof(uint32_t) * n, cudaMemcpyHostToDevice));
         if (I->has_ucd) chk(cudaMemcpy(I->rec_ucd, ru.data(), sizeof(uint32_t) * n, cudaMemcpyHostToDevice));

@@ -84,21 +84,50 @@ __device__ __forceinline__ uint32_t group_ballot(bool pred, int gbase) {
     return (__ballot_sync(kFull, pred) >> gbase) & gmask<G>();
 }
 
+// Inclusive scan over the first LIMIT lanes of each G-lane segment.  One predicated SHFL.UP + add
+// per step: the shuffle's in-range predicate replaces the lane-index compare/select.
 template <int G, int LIMIT = G>
-__device__ __forceinline__ uint32_t group_incl_scan(uint32_t v, int l) {
+__device__ __forceinline__ uint32_t group_incl_scan(uint32_t v, int /*l*/) {
+    constexpr uint32_t c = (uint32_t)(32 - G) << 8;
 #pragma unroll
     for (int off = 1; off < LIMIT; off <<= 1) {
-        const uint32_t y = __shfl_up_sync(kFull, v, off, G);
-        if (l >= off) v += y;
+        asm volatile(
+            "{\n\t.reg .pred p;\n\t.reg .b32 t;\n\t"
+            "shfl.sync.up.b32 t|p, %0, %1, %2, 0xffffffff;\n\t"
+            "@p add.u32 %0, %0, t;\n\t}"
+            : "+r"(v)
+            : "r"(off), "r"(c));
     }
     return v;
 }
 
 template <int G>
 __device__ __forceinline__ int32_t group_sum(int32_t v) {
+    if constexpr (G == 32) {
+        return (int32_t)__reduce_add_sync(kFull, (uint32_t)v);
+    } else {
 #pragma unroll
-    for (int off = G / 2; off > 0; off >>= 1) v += __shfl_xor_sync(kFull, v, off, G);
-    return v;
+        for (int off = G / 2; off > 0; off >>= 1) v += __shfl_xor_sync(kFull, v, off, G);
+        return v;
+    }
+}
+
+// Sum of a lane's E packed records with two independent 3-input add chains.
+template <int E>
+__device__ __forceinline__ uint32_t lane_total(const uint32_t (&r)[E]) {
+    if constexpr (E == 1) {
+        return r[0];
+    } else {
+        uint32_t a0 = 0, a1 = 0;
+#pragma unroll
+        for (int i = 0; i + 1 < E; i += 2) {
+            if ((i >> 1) & 1)
+                a1 += r[i] + r[i + 1];
+            else
+                a0 += r[i] + r[i + 1];
+        }
+        return a0 + a1;
+    }
 }
 
 // highest set bit index (x != 0)
@@ -118,9 +147,7 @@ __device__ __forceinline__ int hibit(uint32_t x) { return 31 - __clz(x); }
 template <int G, int E, class Elem>
 __device__ __forceinline__ int32_t eval_cdd(const uint32_t (&rec)[E], int l, int gbase, int n,
                                             int32_t d, const RecLayout& L, Elem&& elem) {
-    uint32_t tot = 0;
-#pragma unroll
-    for (int i = 0; i < E; ++i) tot += rec[i];
+    const uint32_t tot = lane_total<E>(rec);
     const uint32_t tP = tot & L.pmask;
     const uint32_t tAB = ((tot >> L.sa) & L.amask) | ((tot >> L.sb) << 16);
     const uint32_t iP = group_incl_scan<G>(tP, l);
@@ -171,9 +198,7 @@ __device__ __forceinline__ int32_t eval_cdd(const uint32_t (&rec)[E], int l, int
 template <int G, int E, class Elem>
 __device__ __forceinline__ int32_t eval_ucddcp(const uint32_t (&rec)[E], int l, int gbase, int n,
                                                const RecLayout& L, Elem&& elem) {
-    uint32_t tot = 0;
-#pragma unroll
-    for (int i = 0; i < E; ++i) tot += rec[i];
+    const uint32_t tot = lane_total<E>(rec);
     const uint32_t tAB = (tot & L.amask) | (((tot >> L.sb) & L.bmask) << 16);
     const uint32_t iAB = group_incl_scan<G>(tAB, l);
     const uint32_t ABb = iAB - tAB;

@@ -29,6 +29,13 @@ struct Instance {
     RecLayout lay_cdd{}, lay_ucd{};
     uint32_t* rec_cdd = nullptr;  // device [n] records by job id
     uint32_t* rec_ucd = nullptr;
+    // warp-per-chain (SA / T0 / DPSO) tables by job id: ab = alpha | beta << 16, p (u8);
+    // UCDDCP: m = M (u8), x = P - M (u8), g = gamma (u16)
+    uint32_t* tab_ab = nullptr;
+    uint8_t* tab_p = nullptr;
+    uint8_t* tab_m = nullptr;
+    uint8_t* tab_x = nullptr;
+    uint16_t* tab_g = nullptr;
     int* err = nullptr;                    // device data-error flag
     unsigned long long* best_key = nullptr;  // device packed (penalty << 32 | id)
     int16_t* best_perm = nullptr;          // device [n]
