@@ -133,17 +133,39 @@ CDD_API int sa_t0(cdd_instance *inst, cdd_problem problem, uint64_t seed, int64_
 /* ------------------------------------------------------------------------------------------ */
 /* Discrete PSO (Alg. 2, eq. (3))                                                   */
 /* ------------------------------------------------------------------------------------------ */
+/* Operators (reading R15): F1 swaps two Floyd-sampled positions; F2 keeps the first
+ * c positions (c uniform in [1, n-1]) and appends the other jobs in personal-best order; F3 keeps
+ * the segment [q0, q1] and fills the other positions left to right with the remaining jobs in
+ * swarm-best order.  x' = c (+) f(x) applies f iff rand(0,1) < c. */
 typedef struct {
     cdd_problem problem;
-    int64_t particles;        /* swarm size on this device                                     */
-    int64_t iters;            /* Alg. 2 #Iterations                                            */
-    double w, c1, c2;         /* probabilities of F1 / F2 / F3 in eq. (3) (silent in the paper)  */
+    int64_t particles;        /* particles on this device (one warp each)                        */
+    int64_t iters;            /* Alg. 2 #Iterations                                              */
+    double w, c1, c2;         /* probabilities of F1 / F2 / F3 in eq. (3) (silent in the paper)    */
     uint64_t seed;
-    int64_t *gbest_trace;     /* optional device int64 [iters]: swarm best value at line 5      */
+    uint64_t particle_offset; /* global id of local particle 0 (multi-GPU swarm: rank * particles) */
+    int64_t *gbest_trace;     /* optional device int64 [iters]: swarm best value at line 5 of     */
+                              /* iteration t (device-local unless the caller reduces across GPUs) */
 } dpso_params;
 CDD_API size_t dpso_workspace_size(const cdd_instance *inst, const dpso_params *params);
-/* ASYNC.  Single-device swarm; the final swarm best goes to the instance's best buffers. */
+/* ASYNC.  Whole run on one device (the swarm is this device's particles): lines 1-2, then
+ * `iters` x lines 4-7, then the final best particle into the instance's best buffers. */
 CDD_API int dpso_run(cdd_instance *inst, const dpso_params *params, void *workspace,
+             size_t workspace_bytes, void *stream);
+/* Stepping interface for a swarm spread over several GPUs.  ASYNC each.
+ *   dpso_begin:   lines 1-2 plus the personal/swarm best of iteration 0 (device-local);
+ *   dpso_gbest_ptrs(t): the packed swarm-best key (int64, (value << 32) | global id) and its
+ *                 int16 [n] sequence that iteration t reads -- all-reduce the key (MIN) and
+ *                 broadcast the sequence from the owning rank between dpso_begin / dpso_iterate;
+ *   dpso_iterate(t): lines 6-7 of iteration t and lines 4-5 of iteration t+1;
+ *   dpso_end:     copies the (reduced) swarm best after `iters` iterations to the best buffers. */
+CDD_API int dpso_begin(cdd_instance *inst, const dpso_params *params, void *workspace,
+               size_t workspace_bytes, void *stream);
+CDD_API int dpso_iterate(cdd_instance *inst, const dpso_params *params, void *workspace,
+                 size_t workspace_bytes, int64_t t, void *stream);
+CDD_API int dpso_gbest_ptrs(const cdd_instance *inst, const dpso_params *params, void *workspace,
+                    int64_t t, int64_t **key_dev, int16_t **perm_dev);
+CDD_API int dpso_end(cdd_instance *inst, const dpso_params *params, void *workspace,
              size_t workspace_bytes, void *stream);
 
 /* ------------------------------------------------------------------------------------------ */

@@ -48,7 +48,7 @@ class SaParams(C.Structure):
 class DpsoParams(C.Structure):
     _fields_ = [("problem", C.c_int), ("particles", C.c_int64), ("iters", C.c_int64),
                 ("w", C.c_double), ("c1", C.c_double), ("c2", C.c_double), ("seed", C.c_uint64),
-                ("gbest_trace", C.c_void_p)]
+                ("particle_offset", C.c_uint64), ("gbest_trace", C.c_void_p)]
 
 
 _vp, _i32, _i64, _u64, _sz = C.c_void_p, C.c_int32, C.c_int64, C.c_uint64, C.c_size_t
@@ -65,6 +65,10 @@ _SIGS = {
     "sa_t0": (C.c_int, [_vp, C.c_int, _u64, _i64, _vp, _vp, _sz, _vp]),
     "dpso_workspace_size": (_sz, [_vp, C.POINTER(DpsoParams)]),
     "dpso_run": (C.c_int, [_vp, C.POINTER(DpsoParams), _vp, _sz, _vp]),
+    "dpso_begin": (C.c_int, [_vp, C.POINTER(DpsoParams), _vp, _sz, _vp]),
+    "dpso_iterate": (C.c_int, [_vp, C.POINTER(DpsoParams), _vp, _sz, _i64, _vp]),
+    "dpso_gbest_ptrs": (C.c_int, [_vp, C.POINTER(DpsoParams), _vp, _i64, _vp, _vp]),
+    "dpso_end": (C.c_int, [_vp, C.POINTER(DpsoParams), _vp, _sz, _vp]),
     "best_device_ptrs": (C.c_int, [_vp, _vp, _vp]),
     "best_get": (C.c_int, [_vp, _vp, _vp, _vp, _vp]),
     "cdd_last_error": (C.c_char_p, []),
@@ -248,25 +252,60 @@ def sa_t0(inst: Instance, problem="cdd", seed=0, samples=5000, stream=None):
     return T0
 
 
-def dpso_run(inst: Instance, particles: int, iters: int, problem="cdd", w=0.5, c1=0.5, c2=0.5,
-             seed=0, trace=False, stream=None, workspace=None):
-    """Discrete PSO (Alg. 2, eq. (3)) on one GPU; best into the instance's best buffers."""
-    import torch
+class Dpso:
+    """A DPSO swarm on one GPU (Alg. 2, eq. (3)).  `run()` does the whole single-GPU run; the
+    stepping methods let a caller exchange the swarm best across GPUs between iterations."""
 
-    dev = torch.device("cuda", inst.device)
-    res = {}
-    if trace:
-        res["gbest_trace"] = torch.empty(iters, dtype=torch.int64, device=dev)
-    p = DpsoParams(PROBLEMS[problem], int(particles), int(iters), float(w), float(c1), float(c2),
-                   int(seed), _dptr(res.get("gbest_trace")))
-    need = int(_lib.dpso_workspace_size(inst.handle, C.byref(p)))
-    if need == 0:
-        _check(_lib.dpso_run(inst.handle, C.byref(p), None, 0, None))
-    if workspace is None or workspace.numel() < need:
-        workspace = torch.empty(need, dtype=torch.uint8, device=dev)
-    res["workspace"] = workspace
-    _check(_lib.dpso_run(inst.handle, C.byref(p), workspace.data_ptr(), need, _stream(stream)))
-    return res
+    def __init__(self, inst: Instance, particles: int, iters: int, problem="cdd", w=0.5, c1=0.5,
+                 c2=0.5, seed=0, particle_offset=0, trace=False):
+        import torch
+
+        self.inst = inst
+        dev = torch.device("cuda", inst.device)
+        self.trace = torch.empty(max(iters, 1), dtype=torch.int64, device=dev) if trace else None
+        self.p = DpsoParams(PROBLEMS[problem], int(particles), int(iters), float(w), float(c1),
+                            float(c2), int(seed), int(particle_offset), _dptr(self.trace))
+        need = int(_lib.dpso_workspace_size(inst.handle, C.byref(self.p)))
+        if need == 0:
+            _check(_lib.dpso_run(inst.handle, C.byref(self.p), None, 0, None))
+        self.ws = torch.empty(need, dtype=torch.uint8, device=dev)
+        self.iters = int(iters)
+
+    def _args(self):
+        return self.inst.handle, C.byref(self.p), self.ws.data_ptr(), self.ws.numel()
+
+    def run(self, stream=None):
+        _check(_lib.dpso_run(*self._args(), _stream(stream)))
+        return self
+
+    def begin(self, stream=None):
+        _check(_lib.dpso_begin(*self._args(), _stream(stream)))
+
+    def iterate(self, t, stream=None):
+        h, p, w, nb = self._args()
+        _check(_lib.dpso_iterate(h, p, w, nb, int(t), _stream(stream)))
+
+    def end(self, stream=None):
+        _check(_lib.dpso_end(*self._args(), _stream(stream)))
+
+    def gbest_tensors(self, t):
+        """Torch views of the swarm-best key (int64 [1]) and sequence (int16 [n]) iteration t reads."""
+        import torch
+
+        key = _vp()
+        perm = _vp()
+        _check(_lib.dpso_gbest_ptrs(self.inst.handle, C.byref(self.p), self.ws.data_ptr(), int(t),
+                                    C.byref(key), C.byref(perm)))
+        dev = torch.device("cuda", self.inst.device)
+        return (torch.as_tensor(_CudaArray(key.value, (1,), "<i8"), device=dev),
+                torch.as_tensor(_CudaArray(perm.value, (self.inst.n,), "<i2"), device=dev))
+
+
+def dpso_run(inst: Instance, particles: int, iters: int, problem="cdd", w=0.5, c1=0.5, c2=0.5,
+             seed=0, trace=False, stream=None):
+    """Discrete PSO (Alg. 2, eq. (3)) on one GPU; best into the instance's best buffers."""
+    sw = Dpso(inst, particles, iters, problem, w, c1, c2, seed, 0, trace).run(stream)
+    return {"gbest_trace": sw.trace, "workspace": sw.ws, "swarm": sw}
 
 
 def best_device_ptrs(inst: Instance):

@@ -390,6 +390,9 @@ static int dpso_validate(const cdd_instance* I, const dpso_params* p, cdd::DpsoL
     if (I->n < 2) return fail(CDD_EINVAL, "DPSO needs n >= 2");
     if (p->particles < 1 || p->particles >= (1ll << 31)) return fail(CDD_EINVAL, "particles must be in [1, 2^31)");
     if (p->iters < 0 || p->iters >= (int64_t)UINT32_MAX) return fail(CDD_EINVAL, "iters must be in [0, 2^32)");
+    if (p->particle_offset + (uint64_t)p->particles > (1ull << 32)) return fail(CDD_EINVAL, "particle ids must fit 32 bits");
+    if (!(p->w >= 0 && p->w <= 1 && p->c1 >= 0 && p->c1 <= 1 && p->c2 >= 0 && p->c2 <= 1))
+        return fail(CDD_EINVAL, "w, c1, c2 must be probabilities");
     L->ucd = ucd;
     L->particles = p->particles;
     L->iters = p->iters;
@@ -397,6 +400,7 @@ static int dpso_validate(const cdd_instance* I, const dpso_params* p, cdd::DpsoL
     L->c1 = p->c1;
     L->c2 = p->c2;
     L->seed = p->seed;
+    L->particle_offset = p->particle_offset;
     L->gbest_trace = p->gbest_trace;
     return CDD_OK;
 }
@@ -407,16 +411,68 @@ size_t dpso_workspace_size(const cdd_instance* I, const dpso_params* p) {
     return cdd::dpso_workspace_bytes(*I, L);
 }
 
+static int dpso_prepare(cdd_instance* I, const dpso_params* p, void* ws, size_t ws_bytes,
+                        cdd::DpsoLaunch* L) {
+    int rc = dpso_validate(I, p, L);
+    if (rc != CDD_OK) return rc;
+    const size_t need = cdd::dpso_workspace_bytes(*I, *L);
+    if (!ws || ws_bytes < need)
+        return fail(CDD_ENOMEM, "workspace too small: need " + std::to_string(need) + " bytes");
+    return CDD_OK;
+}
+
 int dpso_run(cdd_instance* I, const dpso_params* p, void* ws, size_t ws_bytes, void* stream) {
+    cdd::DpsoLaunch L{};
+    int rc = dpso_prepare(I, p, ws, ws_bytes, &L);
+    if (rc != CDD_OK) return rc;
+    DeviceGuard g(I->device);
+    cudaStream_t s = as_stream(stream);
+    cudaError_t e = cdd::dpso_begin(*I, L, ws, s);
+    for (int64_t t = 0; e == cudaSuccess && t < L.iters; ++t) e = cdd::dpso_iterate(*I, L, ws, t, s);
+    if (e == cudaSuccess) e = cdd::dpso_end(*I, L, ws, s);
+    if (e != cudaSuccess) return cuda_fail(e, "dpso_run");
+    I->has_best = true;
+    return CDD_OK;
+}
+
+int dpso_begin(cdd_instance* I, const dpso_params* p, void* ws, size_t ws_bytes, void* stream) {
+    cdd::DpsoLaunch L{};
+    int rc = dpso_prepare(I, p, ws, ws_bytes, &L);
+    if (rc != CDD_OK) return rc;
+    DeviceGuard g(I->device);
+    cudaError_t e = cdd::dpso_begin(*I, L, ws, as_stream(stream));
+    return e == cudaSuccess ? CDD_OK : cuda_fail(e, "dpso_begin");
+}
+
+int dpso_iterate(cdd_instance* I, const dpso_params* p, void* ws, size_t ws_bytes, int64_t t,
+                 void* stream) {
+    cdd::DpsoLaunch L{};
+    int rc = dpso_prepare(I, p, ws, ws_bytes, &L);
+    if (rc != CDD_OK) return rc;
+    if (t < 0 || t >= L.iters) return fail(CDD_EINVAL, "t must be in [0, iters)");
+    DeviceGuard g(I->device);
+    cudaError_t e = cdd::dpso_iterate(*I, L, ws, t, as_stream(stream));
+    return e == cudaSuccess ? CDD_OK : cuda_fail(e, "dpso_iterate");
+}
+
+int dpso_gbest_ptrs(const cdd_instance* I, const dpso_params* p, void* ws, int64_t t,
+                    int64_t** key_dev, int16_t** perm_dev) {
     cdd::DpsoLaunch L{};
     int rc = dpso_validate(I, p, &L);
     if (rc != CDD_OK) return rc;
+    if (!ws) return fail(CDD_EINVAL, "workspace is NULL");
+    if (t < 0 || t > L.iters) return fail(CDD_EINVAL, "t must be in [0, iters]");
+    cdd::dpso_gbest(*I, L, ws, t, key_dev, perm_dev);
+    return CDD_OK;
+}
+
+int dpso_end(cdd_instance* I, const dpso_params* p, void* ws, size_t ws_bytes, void* stream) {
+    cdd::DpsoLaunch L{};
+    int rc = dpso_prepare(I, p, ws, ws_bytes, &L);
+    if (rc != CDD_OK) return rc;
     DeviceGuard g(I->device);
-    const size_t need = cdd::dpso_workspace_bytes(*I, L);
-    if (!ws || ws_bytes < need)
-        return fail(CDD_ENOMEM, "workspace too small: need " + std::to_string(need) + " bytes");
-    cudaError_t e = cdd::launch_dpso(*I, L, ws, as_stream(stream));
-    if (e != cudaSuccess) return cuda_fail(e, "dpso_run");
+    cudaError_t e = cdd::dpso_end(*I, L, ws, as_stream(stream));
+    if (e != cudaSuccess) return cuda_fail(e, "dpso_end");
     I->has_best = true;
     return CDD_OK;
 }

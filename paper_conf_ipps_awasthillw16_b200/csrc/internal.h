@@ -73,11 +73,15 @@ struct DpsoLaunch {
     bool ucd;
     int64_t particles, iters;
     double w, c1, c2;
-    uint64_t seed;
+    uint64_t seed, particle_offset;
     int64_t* gbest_trace;
 };
 size_t dpso_workspace_bytes(const Instance& I, const DpsoLaunch& p);
-cudaError_t launch_dpso(Instance& I, const DpsoLaunch& p, void* ws, cudaStream_t s);
+cudaError_t dpso_begin(Instance& I, const DpsoLaunch& p, void* ws, cudaStream_t s);
+cudaError_t dpso_iterate(Instance& I, const DpsoLaunch& p, void* ws, int64_t t, cudaStream_t s);
+void dpso_gbest(const Instance& I, const DpsoLaunch& p, void* ws, int64_t t, int64_t** key,
+                int16_t** perm);
+cudaError_t dpso_end(Instance& I, const DpsoLaunch& p, void* ws, cudaStream_t s);
 
 int sa_e_for_n(int n);  // elements per lane of the warp-per-chain kernels
 

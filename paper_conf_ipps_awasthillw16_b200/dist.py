@@ -35,3 +35,24 @@ def global_best(inst, ids_per_rank: int, group=None) -> int:
     """Reduce the instance's device-resident best (after sa_run / dpso_run) across all ranks."""
     key, perm = best_device_tensors(inst)
     return reduce_best(key, perm, ids_per_rank, group)
+
+
+def dpso_run_distributed(inst, particles_per_rank: int, iters: int, problem="cdd", w=0.5, c1=0.5,
+                         c2=0.5, seed=0, group=None, trace=False):
+    """One swarm spread over all ranks (global particle ids rank*P .. rank*P+P-1).  The swarm best of
+    Alg. 2 line 5 is global every iteration: after each device-local step the packed key is
+    MIN-all-reduced and the winner's sequence broadcast from its owner, then iteration t runs."""
+    from . import Dpso
+
+    rank = dist.get_rank(group)
+    sw = Dpso(inst, particles_per_rank, iters, problem, w, c1, c2, seed,
+              particle_offset=rank * particles_per_rank, trace=trace)
+    sw.begin()
+    for t in range(iters):
+        key, perm = sw.gbest_tensors(t)
+        reduce_best(key, perm, particles_per_rank, group)
+        sw.iterate(t)
+    key, perm = sw.gbest_tensors(iters)
+    reduce_best(key, perm, particles_per_rank, group)
+    sw.end()
+    return sw

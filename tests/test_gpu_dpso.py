@@ -1,0 +1,99 @@
+"""GPU parity: DPSO (Alg. 2, eq. (3)) replayed against the oracle (bit-exact swarm-best traces)."""
+import numpy as np
+import pytest
+
+import gen
+import oracle
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def lib():
+    import torch
+
+    assert torch.cuda.is_available()
+    import paper_conf_ipps_awasthillw16_b200 as m
+
+    return m
+
+
+@pytest.mark.parametrize("n,particles,iters,problem,w,c1,c2", [
+    (10, 64, 50, "cdd", 0.5, 0.5, 0.5),
+    (37, 100, 40, "cdd", 0.3, 0.7, 0.9),
+    (100, 256, 30, "cdd", 0.5, 0.5, 0.5),
+    (200, 96, 20, "ucddcp", 0.5, 0.5, 0.5),
+    (500, 64, 10, "cdd", 1.0, 1.0, 1.0),
+    (1000, 40, 6, "cdd", 0.5, 0.5, 0.5),
+    (60, 50, 20, "cdd", 0.0, 0.0, 0.0),
+])
+def test_dpso_parity(lib, n, particles, iters, problem, w, c1, c2):
+    import torch
+
+    inst = gen.ucddcp_instance(n, 2) if problem == "ucddcp" else gen.cdd_instance(n, 3, 0.6)
+    ins = lib.Instance.from_gen(inst)
+    seed = 4321 + n
+    res = lib.dpso_run(ins, particles, iters, problem=problem, w=w, c1=c1, c2=c2, seed=seed,
+                       trace=True)
+    torch.cuda.synchronize()
+    pen, perm, gid = lib.best_get(ins)
+    pr = oracle.Problem.from_instance(inst)
+    P = oracle.CDD if problem == "cdd" else oracle.UCDDCP
+    ref = oracle.dpso_run(pr, oracle.dpso_params(problem=P, particles=particles, iters=iters, w=w,
+                                                 c1=c1, c2=c2, seed=seed), trace=True)
+    assert np.array_equal(res["gbest_trace"].cpu().numpy()[:iters], ref["gbest_trace"])
+    assert (pen, gid) == (ref["E_best"], ref["id"])
+    assert np.array_equal(perm, ref["best"])
+
+
+def test_dpso_emulated_two_ranks(lib):
+    # the stepping interface with a host-side exchange reproduces the single swarm of 2P particles
+    import torch
+
+    inst = gen.cdd_instance(80, 4, 0.4)
+    P, iters, seed = 48, 12, 99
+    ranks = []
+    for r in range(2):
+        ins = lib.Instance.from_gen(inst)
+        ranks.append((ins, lib.Dpso(ins, P, iters, seed=seed, particle_offset=r * P, trace=True)))
+    for ins, sw in ranks:
+        sw.begin()
+
+    def exchange(t):
+        torch.cuda.synchronize()
+        views = [sw.gbest_tensors(t) for _, sw in ranks]
+        keys = [int(k.item()) for k, _ in views]
+        kmin = min(keys)
+        owner = (kmin & 0xFFFFFFFF) // P
+        win = views[owner][1].clone()
+        for k, p in views:
+            k.fill_(kmin)
+            p.copy_(win)
+        torch.cuda.synchronize()
+
+    for t in range(iters):
+        exchange(t)
+        for _, sw in ranks:
+            sw.iterate(t)
+    exchange(iters)
+    for _, sw in ranks:
+        sw.end()
+    torch.cuda.synchronize()
+    pr = oracle.Problem.from_instance(inst)
+    ref = oracle.dpso_run(pr, oracle.dpso_params(particles=2 * P, iters=iters, seed=seed), trace=True)
+    for ins, sw in ranks:
+        pen, perm, gid = lib.best_get(ins)
+        assert (pen, gid) == (ref["E_best"], ref["id"]) and np.array_equal(perm, ref["best"])
+        assert np.array_equal(sw.trace.cpu().numpy(), ref["gbest_trace"])
+
+
+def test_dpso_n10_reaches_optimum(lib):
+    import json
+    import os
+
+    gold = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "config1.json")))
+    inst = gen.cdd_instance(10, 1, 0.4)
+    ins = lib.Instance.from_gen(inst)
+    lib.dpso_run(ins, 768, 200, seed=5)  # 768 particles as in the paper
+    pen, perm, gid = lib.best_get(ins)
+    assert pen == gold["optimum"]
