@@ -1,0 +1,164 @@
+// sa_group.cuh -- the CDD SA kernel: G lanes per chain, 32/G chains per warp.
+//
+// Differences from the warp-per-chain kernel (sa.cu, used for UCDDCP):
+//  * every warp instruction of the fixed per-step work (move decode, scans, ballots, Metropolis,
+//    bookkeeping) serves 32/G chains at once;
+//  * the per-lane totals of the packed records are kept in shared memory and updated by the
+//    movers with shared atomics (delta of the <= 4 moved positions), so no full pass is needed to
+//    form them; the records are streamed from shared memory once per step (pass 2);
+//  * the job ids of the current sequence live in a per-chain global slot (L2-resident), written
+//    only when a move is accepted.
+// The arithmetic is the evaluator of device_common.cuh / chain.cuh.
+#pragma once
+#include <cuda_runtime.h>
+
+#include <climits>
+
+#include "device_common.cuh"
+#include "internal.h"
+
+namespace cdd {
+
+template <int G, int E>
+struct GChain {
+    static constexpr int NP = G * E;
+    static constexpr int ABS = E >= 8 ? E + 4 : E;                         // words per lane row
+    static constexpr int PS = E == 64 ? 80 : (E == 32 ? 48 : E);            // bytes per lane row
+    static constexpr int SPR = E >= G ? E / G : 1;                         // boundary elements per lane
+    static constexpr int AB_BYTES = G * ABS * 4;
+    static constexpr int P_BYTES = (G * PS + 15) / 16 * 16;
+    static constexpr int TOT_BYTES = G * 8;
+    static constexpr int BYTES = (AB_BYTES + P_BYTES + TOT_BYTES + 15) / 16 * 16;
+    uint8_t* base;
+    __device__ __forceinline__ uint32_t* ab() const { return reinterpret_cast<uint32_t*>(base); }
+    __device__ __forceinline__ uint8_t* pb() const { return base + AB_BYTES; }
+    __device__ __forceinline__ uint2* tot() const { return reinterpret_cast<uint2*>(base + AB_BYTES + P_BYTES); }
+    static __device__ __forceinline__ int ab_w(int k) { return (k / E) * ABS + (k % E); }
+    static __device__ __forceinline__ int pb_b(int k) { return (k / E) * PS + (k % E); }
+};
+
+// Inclusive scan over G-lane segments (predicated shuffle, see device_common.cuh).
+template <int G>
+__device__ __forceinline__ uint32_t gscan(uint32_t v) {
+    return group_incl_scan<G>(v, 0);
+}
+
+template <int G>
+__device__ __forceinline__ uint32_t gsum(uint32_t v) {
+    if constexpr (G == 32) {
+        return __reduce_add_sync(kFull, v);
+    } else {
+#pragma unroll
+        for (int off = G / 2; off > 0; off >>= 1) v += __shfl_xor_sync(kFull, v, off, G);
+        return v;
+    }
+}
+
+// CDD penalty of the group's chain.  tAB / tP: this lane's totals (maintained incrementally).
+template <int G, int E>
+__device__ __forceinline__ int32_t gchain_eval_cdd(const GChain<G, E>& ch, int l, int gbase, int n,
+                                                   int32_t d, uint32_t tAB, uint32_t tP) {
+    using C = GChain<G, E>;
+    constexpr int SPR = C::SPR;
+    const uint32_t iP = gscan<G>(tP);
+    const uint32_t iAB = gscan<G>(tAB);
+    const int32_t Pb = (int32_t)(iP - tP);
+    const uint32_t ABb = iAB - tAB;
+    const int32_t Ab = (int32_t)(ABb & 0xffffu), Bb = (int32_t)(ABb >> 16);
+    const int32_t Btot = (int32_t)(__shfl_sync(kFull, iAB, G - 1, G) >> 16);
+    const bool lane_valid = l * E < n;
+    const int Lk = hibit(group_ballot<G>(lane_valid && (Ab + Bb <= Btot), gbase));
+    const int Lt = hibit(group_ballot<G>(lane_valid && (Pb <= d), gbase));
+    const int Ls = min(Lk, Lt);
+
+    // ---- boundary lane Ls: SPR consecutive elements per lane
+    const int32_t PbS = __shfl_sync(kFull, Pb, Ls, G);
+    const uint32_t ABbS = __shfl_sync(kFull, ABb, Ls, G);
+    const int32_t SbS = (int32_t)(ABbS & 0xffffu) + (int32_t)(ABbS >> 16);
+    const int e0 = l * SPR;  // first element (within the row) of this lane
+    const bool lane_in = e0 < E;
+    uint32_t rv[SPR];
+    uint32_t pv = 0;
+    if constexpr (SPR == 4) {
+        const uint4 x = *reinterpret_cast<const uint4*>(ch.ab() + Ls * C::ABS + e0);
+        rv[0] = x.x; rv[1] = x.y; rv[2] = x.z; rv[3] = x.w;
+        pv = *reinterpret_cast<const uint32_t*>(ch.pb() + Ls * C::PS + e0);
+    } else if constexpr (SPR == 2) {
+        const uint2 x = *reinterpret_cast<const uint2*>(ch.ab() + Ls * C::ABS + e0);
+        rv[0] = x.x; rv[1] = x.y;
+        pv = *reinterpret_cast<const uint16_t*>(ch.pb() + Ls * C::PS + e0);
+    } else {
+        rv[0] = lane_in ? ch.ab()[Ls * C::ABS + e0] : 0u;
+        pv = lane_in ? ch.pb()[Ls * C::PS + e0] : 0u;
+    }
+    uint32_t v[SPR];
+    uint32_t lsum = 0;
+#pragma unroll
+    for (int i = 0; i < SPR; ++i) {
+        const uint32_t pi = (pv >> (8 * i)) & 0xffu;
+        v[i] = pi | (((rv[i] & 0xffffu) + (rv[i] >> 16)) << 16);
+        lsum += v[i];
+    }
+    uint32_t ex = gscan<G>(lsum) - lsum;
+    int32_t Cex[SPR], Sex[SPR], pe[SPR];
+    uint32_t cnt = 0;
+    const int kbase = Ls * E + e0;
+#pragma unroll
+    for (int i = 0; i < SPR; ++i) {
+        Cex[i] = PbS + (int32_t)(ex & 0xffffu);
+        Sex[i] = SbS + (int32_t)(ex >> 16);
+        pe[i] = (int32_t)(v[i] & 0xffffu);
+        const bool ok = lane_in && (kbase + i < n) && (Sex[i] <= Btot);
+        cnt += ok ? 1u : 0u;
+        ex += v[i];
+    }
+    const int ik = (int)gsum<G>(cnt) - 1;  // k0 - Ls*E when Ls == Lk
+    const int own = ik < 0 ? 0 : ik / SPR, ei = ik < 0 ? 0 : ik % SPR;
+    int32_t csel = Cex[0] + pe[0];
+#pragma unroll
+    for (int i = 1; i < SPR; ++i) csel = (ei == i) ? Cex[i] + pe[i] : csel;
+    const int32_t Ck0 = __shfl_sync(kFull, csel, own, G);
+    const int32_t D = (Ls == Lk) ? min(Ck0, d) : d;
+    int32_t corr = 0;
+#pragma unroll
+    for (int i = 0; i < SPR; ++i) {
+        const bool vi = lane_in && (kbase + i < n);
+        corr += vi ? (Sex[i] - Btot) * min(pe[i], max(0, D - Cex[i])) : 0;
+    }
+
+    // ---- F(C_{m'}) streamed: 4 records per LDS.128, p bytes 16 per LDS.128
+    const bool amode = l < Ls;
+    const uint32_t sel = amode ? 0x5410u : 0x7632u;
+    const uint32_t* abr = ch.ab() + l * C::ABS;
+    const uint8_t* pbr = ch.pb() + l * C::PS;
+    uint32_t s = 0, acc = 0;
+#pragma unroll
+    for (int q = 0; q < E / 16 || (q == 0 && E < 16); ++q) {
+        uint32_t pw[4];
+        if constexpr (E >= 16) {
+            const uint4 x = *reinterpret_cast<const uint4*>(pbr + 16 * q);
+            pw[0] = x.x; pw[1] = x.y; pw[2] = x.z; pw[3] = x.w;
+        } else if constexpr (E == 8) {
+            const uint2 x = *reinterpret_cast<const uint2*>(pbr);
+            pw[0] = x.x; pw[1] = x.y; pw[2] = 0; pw[3] = 0;
+        } else {
+            pw[0] = *reinterpret_cast<const uint32_t*>(pbr);
+            pw[1] = pw[2] = pw[3] = 0;
+        }
+#pragma unroll
+        for (int v4 = 0; v4 < 4 && 16 * q + 4 * v4 < E; ++v4) {
+            const uint4 r = *reinterpret_cast<const uint4*>(abr + 16 * q + 4 * v4);
+            uint32_t t = s + r.x;
+            acc = __dp2a_lo(__byte_perm(s, t, sel), pw[v4], acc);
+            s = t + r.y;
+            t = s + r.z;
+            acc = __dp2a_hi(__byte_perm(s, t, sel), pw[v4], acc);
+            s = t + r.w;
+        }
+    }
+    const int32_t base = amode ? Ab : (Btot - Bb);
+    const int32_t contrib = base * (int32_t)tP + (amode ? (int32_t)acc : -(int32_t)acc) + corr;
+    return (int32_t)gsum<G>((uint32_t)contrib);
+}
+
+}  // namespace cdd
