@@ -60,6 +60,28 @@ __device__ __forceinline__ int32_t gchain_eval_cdd(const GChain<G, E>& ch, int l
                                                    int32_t d, uint32_t tAB, uint32_t tP) {
     using C = GChain<G, E>;
     constexpr int SPR = C::SPR;
+    // pass-2 operands are loaded first so their latency hides behind the scans and the spread
+    const uint32_t* abr = ch.ab() + l * C::ABS;
+    const uint8_t* pbr = ch.pb() + l * C::PS;
+    uint32_t rr[E];
+    uint32_t pw[E / 4];
+#pragma unroll
+    for (int v = 0; v < E / 4; ++v) {
+        const uint4 x = *reinterpret_cast<const uint4*>(abr + 4 * v);
+        rr[4 * v] = x.x; rr[4 * v + 1] = x.y; rr[4 * v + 2] = x.z; rr[4 * v + 3] = x.w;
+    }
+    if constexpr (E >= 16) {
+#pragma unroll
+        for (int q = 0; q < E / 16; ++q) {
+            const uint4 x = *reinterpret_cast<const uint4*>(pbr + 16 * q);
+            pw[4 * q] = x.x; pw[4 * q + 1] = x.y; pw[4 * q + 2] = x.z; pw[4 * q + 3] = x.w;
+        }
+    } else if constexpr (E == 8) {
+        const uint2 x = *reinterpret_cast<const uint2*>(pbr);
+        pw[0] = x.x; pw[1] = x.y;
+    } else {
+        pw[0] = *reinterpret_cast<const uint32_t*>(pbr);
+    }
     const uint32_t iP = gscan<G>(tP);
     const uint32_t iAB = gscan<G>(tAB);
     const int32_t Pb = (int32_t)(iP - tP);
@@ -126,35 +148,16 @@ __device__ __forceinline__ int32_t gchain_eval_cdd(const GChain<G, E>& ch, int l
         corr += vi ? (Sex[i] - Btot) * min(pe[i], max(0, D - Cex[i])) : 0;
     }
 
-    // ---- F(C_{m'}) streamed: 4 records per LDS.128, p bytes 16 per LDS.128
+    // ---- F(C_{m'}): two positions per PRMT (16-bit prefix halves) + IDP.2A (x 8-bit p)
     const bool amode = l < Ls;
     const uint32_t sel = amode ? 0x5410u : 0x7632u;
-    const uint32_t* abr = ch.ab() + l * C::ABS;
-    const uint8_t* pbr = ch.pb() + l * C::PS;
     uint32_t s = 0, acc = 0;
 #pragma unroll
-    for (int q = 0; q < E / 16 || (q == 0 && E < 16); ++q) {
-        uint32_t pw[4];
-        if constexpr (E >= 16) {
-            const uint4 x = *reinterpret_cast<const uint4*>(pbr + 16 * q);
-            pw[0] = x.x; pw[1] = x.y; pw[2] = x.z; pw[3] = x.w;
-        } else if constexpr (E == 8) {
-            const uint2 x = *reinterpret_cast<const uint2*>(pbr);
-            pw[0] = x.x; pw[1] = x.y; pw[2] = 0; pw[3] = 0;
-        } else {
-            pw[0] = *reinterpret_cast<const uint32_t*>(pbr);
-            pw[1] = pw[2] = pw[3] = 0;
-        }
-#pragma unroll
-        for (int v4 = 0; v4 < 4 && 16 * q + 4 * v4 < E; ++v4) {
-            const uint4 r = *reinterpret_cast<const uint4*>(abr + 16 * q + 4 * v4);
-            uint32_t t = s + r.x;
-            acc = __dp2a_lo(__byte_perm(s, t, sel), pw[v4], acc);
-            s = t + r.y;
-            t = s + r.z;
-            acc = __dp2a_hi(__byte_perm(s, t, sel), pw[v4], acc);
-            s = t + r.w;
-        }
+    for (int j = 0; j < E; j += 2) {
+        const uint32_t t = s + rr[j];
+        acc = (j & 2) ? __dp2a_hi(__byte_perm(s, t, sel), pw[j >> 2], acc)
+                      : __dp2a_lo(__byte_perm(s, t, sel), pw[j >> 2], acc);
+        s = t + rr[j + 1];
     }
     const int32_t base = amode ? Ab : (Btot - Bb);
     const int32_t contrib = base * (int32_t)tP + (amode ? (int32_t)acc : -(int32_t)acc) + corr;
