@@ -79,8 +79,9 @@ CDD_API int cdd_instance_query(const cdd_instance *inst, int32_t *n, int64_t *d,
 /* ------------------------------------------------------------------------------------------ */
 /* ASYNC.  out[b] (device int64) = optimal eq. (1) penalty of sequence row b for the CDD with the
  * instance's d (restrictive or not) -- the value the linear algorithm of P:94-122 finds.
- * perms: device int16 [batch][ld].  A job id outside [0,n) is treated as an empty job and raises
- * the instance's data-error flag (see cdd_check); duplicates are not detected. */
+ * perms: device int16 [batch][ld].  A job id outside [0,n) raises the instance's data-error flag
+ * (see cdd_check) and makes that row's penalty unspecified; nothing is read out of bounds.
+ * Duplicates are not detected. */
 CDD_API int cdd_eval_batch(cdd_instance *inst, const int16_t *perms, int64_t ld, int64_t batch,
                    int64_t *out, void *stream);
 /* ASYNC.  As above for the UCDDCP objective eq. (2).  CDD_EINVAL if the instance has
