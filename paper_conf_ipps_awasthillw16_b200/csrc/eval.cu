@@ -72,7 +72,7 @@ __device__ __forceinline__ void load_words(const int16_t* __restrict__ row, int 
 }
 
 #ifndef CDD_EVAL_MIN_BLOCKS
-#define CDD_EVAL_MIN_BLOCKS 3
+#define CDD_EVAL_MIN_BLOCKS 2
 #endif
 template <int G, int E, bool UCD, bool VEC>
 __global__ void __launch_bounds__(kEvalThreads, CDD_EVAL_MIN_BLOCKS) eval_batch_kernel(
