@@ -121,8 +121,9 @@ def random_small(n: int, seed: int, pmax: int = 6, wmax: int = 5, h: float | Non
 # Job sequences
 # --------------------------------------------------------------------------------------------
 def pad_ld(n: int) -> int:
-    """Row stride (elements) for int16 sequence batches: a multiple of 8 (16-byte rows)."""
-    return (n + 7) // 8 * 8
+    """Row stride (elements) for int16 sequence batches: a multiple of 16 (32-byte rows, which
+    lets the evaluator use 256-bit loads)."""
+    return (n + 15) // 16 * 16
 
 
 def random_perms(batch: int, n: int, seed: int, ld: int | None = None) -> np.ndarray:

@@ -125,6 +125,21 @@ def test_unaligned_and_odd_stride(lib):
     assert np.array_equal(lib.cdd_eval_batch(ins, un).cpu().numpy(), _oracle(inst, p8))
 
 
+@pytest.mark.parametrize("n", [513, 600, 777, 1000, 1001, 1016, 1023, 1024])
+@pytest.mark.parametrize("pad", [0, 3, 8, 16])
+def test_large_n_row_strides(lib, n, pad):
+    # 512 < n <= 1024 uses the 64-unit kernel: 256-bit loads when ld % 16 == 0, 128-bit when
+    # ld % 8 == 0, scalar otherwise; straddling vectors when n % 8 != 0
+    ld = n + pad
+    if ld % 8 == 0 or pad == 3:
+        inst = gen.cdd_instance(n, 2, 0.4)
+        perms = gen.random_perms(333, n, n + pad, ld=ld)
+        perms[:, n:] = 12345  # garbage past n must be ignored
+        for h in (0.2, 0.8):
+            d = int(h * inst.sum_p)
+            assert np.array_equal(_gpu_eval(lib, inst, perms, d=d), _oracle(inst, perms, d=d)), (n, ld, h)
+
+
 def test_invalid_ids_flagged(lib):
     inst = gen.cdd_instance(50, 1, 0.4)
     perms = gen.random_perms(10, 50, 1)
