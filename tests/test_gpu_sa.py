@@ -87,13 +87,15 @@ def test_many_chains_trace_parity(lib, n, chains, steps):
     assert np.array_equal(perm, full["best"])
 
 
-def test_ucddcp_sa_parity(lib):
-    inst = gen.ucddcp_instance(200, 4)
-    ins, res, (pen, perm, gid), pr, p, T0 = _run_both(lib, inst, "ucddcp", 48, 400, 77,
+@pytest.mark.parametrize("n,chains,steps", [(40, 32, 300), (200, 48, 400), (333, 40, 200),
+                                            (1000, 20, 150)])
+def test_ucddcp_sa_parity(lib, n, chains, steps):
+    inst = gen.ucddcp_instance(n, 4)
+    ins, res, (pen, perm, gid), pr, p, T0 = _run_both(lib, inst, "ucddcp", chains, steps, 77,
                                                      samples=600)
     cb = res["chain_best"].cpu().numpy()
     tr = res["trace"].cpu().numpy()
-    for c in range(48):
+    for c in range(chains):
         ref = oracle.sa_chain(pr, p, T0, c, trace=True)
         assert np.array_equal(tr[c] >> 1, ref["E_new"]) and cb[c] == ref["E_best"], c
     full = oracle.sa_run(pr, p, T0)
