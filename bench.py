@@ -186,6 +186,7 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-eval", action="store_true")
+    ap.add_argument("--no-configs", action="store_true")
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)
@@ -297,6 +298,8 @@ def main():
     extra = {}
     if rank == 0 and not args.no_eval:
         extra["eval_batch"] = bench_eval(lib, gens[1], dev, stream, peaks)
+    if rank == 0 and not args.no_configs:
+        extra["other_configs"] = bench_configs(lib, dev, stream)
     e2e = None
     if not args.no_e2e:
         e2e = bench_e2e(lib, gens, chains, steps, rank, world, dev, stream, max(1, args.steps // 2))
@@ -321,6 +324,75 @@ def main():
         print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()
+
+
+def _timed(stream, fn, reps=1):
+    import torch
+
+    fn()  # warm-up (JIT of nothing, but allocations and first-launch costs)
+    torch.cuda.synchronize()
+    e1 = torch.cuda.Event(enable_timing=True)
+    e2 = torch.cuda.Event(enable_timing=True)
+    e1.record(stream)
+    for _ in range(reps):
+        fn()
+    e2.record(stream)
+    torch.cuda.synchronize()
+    return e1.elapsed_time(e2) / reps / 1000.0
+
+
+def bench_configs(lib, dev, stream):
+    """Device throughput on the other BASELINE configs (one line each; CUDA-event timed)."""
+    import torch
+
+    import gen
+
+    out = {}
+    # config 1: CDD n=10, h=0.4, seed 1 -- all 10! sequences + one 10k-step chain
+    g1 = gen.cdd_instance(10, 1, 0.4)
+    i1 = lib.Instance.from_gen(g1, device=dev.index)
+    allp = torch.from_numpy(gen.all_perms(10)).to(dev)
+    o1 = torch.empty(allp.shape[0], dtype=torch.int64, device=dev)
+    t = _timed(stream, lambda: lib.cdd_eval_batch(i1, allp, o1), reps=5)
+    t_sa = _timed(stream, lambda: lib.sa_run(i1, 1, 10000, seed=0x5EED0001))
+    pen, _, _ = lib.best_get(i1)
+    out["config1"] = {"exhaustive_evals_per_s": allp.shape[0] / t, "exhaustive_ms": 1000 * t,
+                      "optimum": int(o1.min().item()), "sa_10k_chain_ms": 1000 * t_sa,
+                      "sa_best": pen}
+    # config 2: CDD n=100, h in {0.2..0.8} (instance 1): 1M random sequences + 4096 chains x 5000
+    p2 = gen.random_perms_device(1 << 20, 100, 2, device=dev)
+    o2 = torch.empty(p2.shape[0], dtype=torch.int64, device=dev)
+    ev, sa = [], []
+    for h in HS:
+        ins = lib.Instance.from_gen(gen.cdd_instance(100, 1, h), device=dev.index)
+        ev.append(p2.shape[0] / _timed(stream, lambda: lib.cdd_eval_batch(ins, p2, o2), reps=10))
+        ws = lib.sa_run(ins, 4096, 5000, seed=0x5EED0002)["workspace"]
+        dt = _timed(stream, lambda: lib.sa_run(ins, 4096, 5000, seed=0x5EED0002, workspace=ws))
+        sa.append(4096 * 5001 / dt)
+    out["config2"] = {"eval_batch_evals_per_s": sum(ev) / len(ev), "sa_evals_per_s": sum(sa) / len(sa),
+                      "workload": "n=100, 4 h x instance 1; 2^20 random sequences; 4096 chains x 5000 steps"}
+    # config 3: UCDDCP n=200 unrestricted, 16384 chains x 5000 steps
+    i3 = lib.Instance.from_gen(gen.ucddcp_instance(200, 1), device=dev.index)
+    ws = lib.sa_run(i3, 16384, 5000, problem="ucddcp", seed=0x5EED0003)["workspace"]
+    dt = _timed(stream, lambda: lib.sa_run(i3, 16384, 5000, problem="ucddcp", seed=0x5EED0003,
+                                           workspace=ws))
+    out["config3"] = {"sa_evals_per_s": 16384 * 5001 / dt, "ms": 1000 * dt,
+                      "workload": "UCDDCP n=200 (d = sum p), 16384 chains x 5000 steps"}
+    # config 4: CDD n=500, h=0.6: DPSO 8192 particles vs SA at equal wall time (1 GPU)
+    i4 = lib.Instance.from_gen(gen.cdd_instance(500, 1, 0.6), device=dev.index)
+    iters = 200
+    sw = lib.Dpso(i4, 8192, iters, seed=0x5EED0004)
+    dt = _timed(stream, lambda: sw.run())
+    dpso_best, _, _ = lib.best_get(i4)
+    sa_rate_steps = 8192 * 200 / _timed(stream, lambda: lib.sa_run(i4, 8192, 200, seed=0x5EED0004))
+    sa_steps = max(1, int(dt * sa_rate_steps / 8192))
+    lib.sa_run(i4, 8192, sa_steps, seed=0x5EED0004)
+    sa_best, _, _ = lib.best_get(i4)
+    out["config4"] = {"dpso_particle_evals_per_s": 8192 * (iters + 1) / dt, "dpso_ms": 1000 * dt,
+                      "dpso_best": dpso_best, "sa_steps_equal_time": sa_steps, "sa_best": sa_best,
+                      "workload": "CDD n=500 h=0.6, DPSO 8192 particles x 200 iterations (w=c1=c2=0.5) vs "
+                                  "8192 SA chains for the same wall time, 1 GPU"}
+    return out
 
 
 def bench_eval(lib, g, dev, stream, peaks, batch=1 << 20, reps=20):
