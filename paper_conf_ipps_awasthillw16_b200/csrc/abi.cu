@@ -62,6 +62,7 @@ void free_instance(cdd_instance* I) {
     cudaFree(I->rec_cdd);
     cudaFree(I->rec_ucd);
     cudaFree(I->tab_ab);
+    cudaFree(I->tab_ab16);
     cudaFree(I->tab_p);
     cudaFree(I->tab_m);
     cudaFree(I->tab_x);
@@ -183,6 +184,12 @@ int cdd_instance_create(int32_t n, const int32_t* p, const int32_t* alpha, const
     }
     chk(cudaMalloc(&I->tab_ab, sizeof(uint32_t) * n));
     chk(cudaMalloc(&I->tab_p, n));
+    I->ab16_ok = amax <= 255 && bmax <= 255;
+    std::vector<uint16_t> tab16(n);
+    for (int i = 0; i < n; ++i) tab16[i] = (uint16_t)((alpha[i] & 0xff) | ((beta[i] & 0xff) << 8));
+    chk(cudaMalloc(&I->tab_ab16, sizeof(uint16_t) * n));
+    if (e == cudaSuccess)
+        chk(cudaMemcpy(I->tab_ab16, tab16.data(), sizeof(uint16_t) * n, cudaMemcpyHostToDevice));
     if (I->has_ucd) {
         chk(cudaMalloc(&I->tab_m, n));
         chk(cudaMalloc(&I->tab_x, n));

@@ -32,6 +32,8 @@ struct Instance {
     // warp-per-chain (SA / T0 / DPSO) tables by job id: ab = alpha | beta << 16, p (u8);
     // UCDDCP: m = M (u8), x = P - M (u8), g = gamma (u16)
     uint32_t* tab_ab = nullptr;
+    uint16_t* tab_ab16 = nullptr;  // alpha | beta << 8 (only when both <= 255: ab16_ok)
+    bool ab16_ok = false;
     uint8_t* tab_p = nullptr;
     uint8_t* tab_m = nullptr;
     uint8_t* tab_x = nullptr;
