@@ -22,6 +22,12 @@
 #include "device_common.cuh"
 #include "internal.h"
 
+// 1: the CDD pass-2 records are loaded into registers before the scans (latency hidden by ILP);
+// 0: streamed in chunks of 16 positions (fewer registers, more resident warps)
+#ifndef CDD_SAG_PREFETCH
+#define CDD_SAG_PREFETCH 0
+#endif
+
 namespace cdd {
 
 // One chain of G lanes x E positions.  ab = alpha | beta << 8 (u16), pb = P (CDD) or M (UCDDCP)
@@ -127,11 +133,13 @@ __device__ __forceinline__ int32_t gchain_eval_cdd(const GChain<G, E>& ch, int l
                                                    int32_t d, uint32_t tAB, uint32_t tP) {
     using C = GChain<G, E>;
     constexpr int SPR = C::SPR;
+#if CDD_SAG_PREFETCH
     // pass-2 operands are loaded first so their latency hides behind the scans and the spread
     uint32_t rr[E / 2];
     uint32_t pw[E / 4];
     load_ab16<E>(reinterpret_cast<const uint8_t*>(ch.ab()) + l * C::AS, rr);
     load_b8<E>(ch.pb() + l * C::PS, pw);
+#endif
     const uint32_t iP = gscan<G>(tP);
     const uint32_t iAB = gscan<G>(tAB);
     const int32_t Pb = (int32_t)(iP - tP);
@@ -194,12 +202,30 @@ __device__ __forceinline__ int32_t gchain_eval_cdd(const GChain<G, E>& ch, int l
     const uint32_t psel = amode ? 0x4044u : 0x4144u;
     const uint32_t wsum = amode ? 0x00010001u : 0x01000100u;
     uint32_t s = 0, acc = 0;
+#if CDD_SAG_PREFETCH
 #pragma unroll
     for (int j = 0; j < E / 2; ++j) {
         const uint32_t f2 = s * 0x10001u + __byte_perm(rr[j], 0u, psel);
         acc = (j & 1) ? __dp2a_hi(f2, pw[j >> 1], acc) : __dp2a_lo(f2, pw[j >> 1], acc);
         s = __dp4a(rr[j], wsum, s);
     }
+#else
+    const uint8_t* arow = reinterpret_cast<const uint8_t*>(ch.ab()) + l * C::AS;
+    const uint8_t* prow = ch.pb() + l * C::PS;
+    constexpr int CH = E >= 16 ? 16 : E;  // positions per chunk
+#pragma unroll
+    for (int c0 = 0; c0 < E; c0 += CH) {
+        uint32_t r[CH / 2], q[CH / 4];
+        load_ab16<CH>(arow + 2 * c0, r);
+        load_b8<CH>(prow + c0, q);
+#pragma unroll
+        for (int j = 0; j < CH / 2; ++j) {
+            const uint32_t f2 = s * 0x10001u + __byte_perm(r[j], 0u, psel);
+            acc = (j & 1) ? __dp2a_hi(f2, q[j >> 1], acc) : __dp2a_lo(f2, q[j >> 1], acc);
+            s = __dp4a(r[j], wsum, s);
+        }
+    }
+#endif
     const int32_t base = amode ? Ab : (Btot - Bb);
     const int32_t contrib = base * (int32_t)tP + (amode ? (int32_t)acc : -(int32_t)acc) + corr;
     return (int32_t)gsum<G>((uint32_t)contrib);
@@ -212,11 +238,13 @@ __device__ __forceinline__ int32_t gchain_eval_ucddcp(const GChain<G, E, true>& 
                                                       int n, uint32_t tAB) {
     using C = GChain<G, E, true>;
     constexpr int SPR = C::SPR;
+#if CDD_SAG_PREFETCH
     uint32_t rr[E / 2], mw[E / 4], xw[E / 4], gw[E / 2];
     load_ab16<E>(reinterpret_cast<const uint8_t*>(ch.ab()) + l * C::AS, rr);
     load_b8<E>(ch.pb() + l * C::PS, mw);
     load_b8<E>(ch.xb() + l * C::PS, xw);
     load_ab16<E>(reinterpret_cast<const uint8_t*>(ch.gh()) + l * C::GS, gw);
+#endif
     const uint32_t iAB = gscan<G>(tAB);
     const uint32_t ABb = iAB - tAB;
     const int32_t Ab = (int32_t)(ABb & 0xffffu), Bb = (int32_t)(ABb >> 16);
@@ -270,6 +298,7 @@ __device__ __forceinline__ int32_t gchain_eval_ucddcp(const GChain<G, E, true>& 
     const uint32_t psel = amode ? 0x4044u : 0x4144u;
     const uint32_t wsum = amode ? 0x00010001u : 0x01000100u;
     uint32_t s = 0, acc = 0;
+#if CDD_SAG_PREFETCH
 #pragma unroll
     for (int j = 0; j < E / 2; ++j) {
         const uint32_t f2 = s * 0x10001u + __byte_perm(rr[j], 0u, psel);
@@ -284,6 +313,35 @@ __device__ __forceinline__ int32_t gchain_eval_ucddcp(const GChain<G, E, true>& 
         }
         s = __dp4a(rr[j], wsum, s);
     }
+#else
+    const uint8_t* arow = reinterpret_cast<const uint8_t*>(ch.ab()) + l * C::AS;
+    const uint8_t* grow = reinterpret_cast<const uint8_t*>(ch.gh()) + l * C::GS;
+    const uint8_t* mrow = ch.pb() + l * C::PS;
+    const uint8_t* xrow = ch.xb() + l * C::PS;
+    constexpr int CH = E >= 16 ? 16 : E;  // positions per chunk
+#pragma unroll
+    for (int c0 = 0; c0 < E; c0 += CH) {
+        uint32_t r[CH / 2], g2[CH / 2], mq[CH / 4], xq[CH / 4];
+        load_ab16<CH>(arow + 2 * c0, r);
+        load_ab16<CH>(grow + 2 * c0, g2);
+        load_b8<CH>(mrow + c0, mq);
+        load_b8<CH>(xrow + c0, xq);
+#pragma unroll
+        for (int j = 0; j < CH / 2; ++j) {
+            const uint32_t f2 = s * 0x10001u + __byte_perm(r[j], 0u, psel);
+            const uint32_t w2 = f2 * sgn + base2;
+            const uint32_t mn2 = __vminu2(w2, g2[j]);
+            if (j & 1) {
+                acc = __dp2a_hi(w2, mq[j >> 1], acc);
+                acc = __dp2a_hi(mn2, xq[j >> 1], acc);
+            } else {
+                acc = __dp2a_lo(w2, mq[j >> 1], acc);
+                acc = __dp2a_lo(mn2, xq[j >> 1], acc);
+            }
+            s = __dp4a(r[j], wsum, s);
+        }
+    }
+#endif
     return (int32_t)gsum<G>(acc + (uint32_t)corr);
 }
 
