@@ -103,6 +103,21 @@ def table1() -> Instance:
     return Instance(5, P, alpha, beta, M, gamma, 16, 0, None, "table1")
 
 
+def ranged_instance(n: int, seed: int, p: tuple, alpha: tuple, beta: tuple, h: float,
+                    problem: str = "cdd") -> Instance:
+    """Instance with chosen value ranges (inclusive) for edge-case tests: large processing times
+    (sum p > 2^16), zero or large penalties (up to 255), d = floor(h * sum p)."""
+    P = _uniform_int(_words(seed, n, 21, n), p[0], p[1])
+    a = _uniform_int(_words(seed, n, 22, n), alpha[0], alpha[1])
+    b = _uniform_int(_words(seed, n, 23, n), beta[0], beta[1])
+    x = _uniform_int(_words(seed, n, 24, n), 0, P // 2)
+    gamma = _uniform_int(_words(seed, n, 25, n), max(alpha[0], 1), max(alpha[1], 1))
+    d = int(math.floor(h * int(P.sum())))
+    if problem == "ucddcp":
+        d = int(P.sum())
+    return Instance(n, P, a, b, (P - x).astype(np.int32), gamma, d, seed, h, problem)
+
+
 def random_small(n: int, seed: int, pmax: int = 6, wmax: int = 5, h: float | None = None,
                  zero_weights: bool = False) -> Instance:
     """Tiny instances with small values for brute-force pins (optionally zero penalties)."""

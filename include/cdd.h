@@ -65,7 +65,9 @@ typedef struct cdd_instance cdd_instance; /* opaque, library-owned, bound to one
  * not fit the packed 32-bit job records of this build (sum alpha, sum beta < 2^16;
  * (sum alpha + sum beta) * sum p < 2^31; field widths for 32 elements per lane <= 32 bits) --
  * always true for the Biskup-Feldmann ranges p<=20, alpha<=10, beta<=15 at n <= 1000.
- * Synchronous.  *out receives the instance. */
+ * If m/gamma are given but the UCDDCP record (alpha, beta for 32 elements, M, P-M, gamma) does
+ * not fit 32 bits, the instance is still created for the CDD and flags bit0 stays clear; the
+ * UCDDCP entry points then return CDD_EINVAL.  Synchronous.  *out receives the instance. */
 CDD_API int cdd_instance_create(int32_t n, const int32_t *p, const int32_t *alpha, const int32_t *beta,
                         const int32_t *m, const int32_t *gamma, int64_t d, int device,
                         cdd_instance **out);

@@ -127,6 +127,13 @@ class Instance:
     def from_gen(cls, inst, device=0):
         return cls(inst.P, inst.alpha, inst.beta, inst.d, inst.M, inst.gamma, device)
 
+    def query(self):
+        """cdd_instance_query: dict(n, d, sum_p, has_ucddcp, unrestricted)."""
+        n, d, sp, fl = C.c_int32(), C.c_int64(), C.c_int64(), C.c_int32()
+        _check(_lib.cdd_instance_query(self.handle, C.byref(n), C.byref(d), C.byref(sp), C.byref(fl)))
+        return dict(n=n.value, d=d.value, sum_p=sp.value, has_ucddcp=bool(fl.value & 1),
+                    unrestricted=bool(fl.value & 2))
+
     @property
     def handle(self):
         if self._h is None:

@@ -155,10 +155,7 @@ int cdd_instance_create(int32_t n, const int32_t* p, const int32_t* alpha, const
             for (int i = 0; i < n; ++i)
                 ru[i] = (uint32_t)alpha[i] | ((uint32_t)beta[i] << L.sb) | ((uint32_t)m[i] << L.sm) |
                         ((uint32_t)(p[i] - m[i]) << L.sx) | ((uint32_t)gamma[i] << L.sg);
-        } else {
-            delete I;
-            return fail(CDD_ERANGE, "UCDDCP data too large for 32-bit packed records");
-        }
+        }  // else: CDD only (flags bit0 clear), the UCDDCP entry points refuse the instance
     }
     DeviceGuard g(device);
     cudaError_t e = cudaSuccess;
@@ -247,7 +244,7 @@ static int eval_common(cdd_instance* I, bool ucd, const int16_t* perms, int64_t 
                        int64_t* out, void* stream) {
     int rc = check_batch_args(I, perms, ld, batch, out);
     if (rc != CDD_OK) return rc;
-    if (ucd && !I->has_ucd) return fail(CDD_EINVAL, "instance has no m/gamma (UCDDCP data)");
+    if (ucd && !I->has_ucd) return fail(CDD_EINVAL, "instance has no UCDDCP data (m/gamma not given or too large for the packed records)");
     if (ucd && I->d < I->sum_p) return fail(CDD_EINVAL, "UCDDCP needs d >= sum p (unrestricted case, P:126)");
     DeviceGuard g(I->device);
     cudaError_t e = cdd::launch_eval_batch(*I, ucd, perms, ld, batch, out, as_stream(stream));
@@ -270,7 +267,7 @@ int cdd_eval_batch_host(cdd_instance* I, cdd_problem problem, const int16_t* per
     if (rc != CDD_OK) return rc;
     if (problem != CDD_PROBLEM_CDD && problem != CDD_PROBLEM_UCDDCP) return fail(CDD_EINVAL, "bad problem");
     const bool ucd = problem == CDD_PROBLEM_UCDDCP;
-    if (ucd && (!I->has_ucd || I->d < I->sum_p)) return fail(CDD_EINVAL, "instance not usable for UCDDCP");
+    if (ucd && (!I->has_ucd || I->d < I->sum_p)) return fail(CDD_EINVAL, "instance not usable for UCDDCP (no m/gamma, data too large for the packed records, or d < sum p)");
     DeviceGuard g(I->device);
     cudaStream_t s = as_stream(stream);
     const int64_t chunk = std::max<int64_t>(1, std::min<int64_t>(batch, (int64_t)(256ll << 20) / (ld * 2)));
@@ -318,7 +315,7 @@ static int sa_validate(const cdd_instance* I, const sa_params* p, cdd::SaLaunch*
     if (!I || !p) return fail(CDD_EINVAL, "instance/params is NULL");
     if (p->problem != CDD_PROBLEM_CDD && p->problem != CDD_PROBLEM_UCDDCP) return fail(CDD_EINVAL, "bad problem");
     const bool ucd = p->problem == CDD_PROBLEM_UCDDCP;
-    if (ucd && (!I->has_ucd || I->d < I->sum_p)) return fail(CDD_EINVAL, "instance not usable for UCDDCP");
+    if (ucd && (!I->has_ucd || I->d < I->sum_p)) return fail(CDD_EINVAL, "instance not usable for UCDDCP (no m/gamma, data too large for the packed records, or d < sum p)");
     if (p->chains < 1) return fail(CDD_EINVAL, "chains must be >= 1");
     if (p->steps < 0 || p->steps >= (int64_t)UINT32_MAX) return fail(CDD_EINVAL, "steps must be in [0, 2^32)");
     if (p->chain_offset + (uint64_t)p->chains > (1ull << 32)) return fail(CDD_EINVAL, "chain ids must fit 32 bits");
@@ -393,7 +390,7 @@ static int dpso_validate(const cdd_instance* I, const dpso_params* p, cdd::DpsoL
     if (!I || !p) return fail(CDD_EINVAL, "instance/params is NULL");
     if (p->problem != CDD_PROBLEM_CDD && p->problem != CDD_PROBLEM_UCDDCP) return fail(CDD_EINVAL, "bad problem");
     const bool ucd = p->problem == CDD_PROBLEM_UCDDCP;
-    if (ucd && (!I->has_ucd || I->d < I->sum_p)) return fail(CDD_EINVAL, "instance not usable for UCDDCP");
+    if (ucd && (!I->has_ucd || I->d < I->sum_p)) return fail(CDD_EINVAL, "instance not usable for UCDDCP (no m/gamma, data too large for the packed records, or d < sum p)");
     if (I->n < 2) return fail(CDD_EINVAL, "DPSO needs n >= 2");
     if (p->particles < 1 || p->particles >= (1ll << 31)) return fail(CDD_EINVAL, "particles must be in [1, 2^31)");
     if (p->iters < 0 || p->iters >= (int64_t)UINT32_MAX) return fail(CDD_EINVAL, "iters must be in [0, 2^32)");

@@ -155,6 +155,11 @@ __device__ __forceinline__ int32_t gchain_eval_cdd(const GChain<G, E>& ch, int l
     const int32_t PbS = __shfl_sync(kFull, Pb, Ls, G);
     const uint32_t ABbS = __shfl_sync(kFull, ABb, Ls, G);
     const int32_t SbS = (int32_t)(ABbS & 0xffffu) + (int32_t)(ABbS >> 16);
+    // Everything below is relative to the start of the row: C - PbS and S - SbS, both < 2^15 per
+    // row (E * 255, E * 510), so they travel packed as c | s << 16.  thr = Btot - SbS >= 0 since
+    // Ls <= Lk.  Padded positions (k >= n) hold zero records: they add nothing to c or s, and where
+    // they pass the S <= Btot test (only if every alpha is 0) they repeat C_n, so no index test.
+    const int32_t thr = Btot - SbS;
     const int e0 = l * SPR;
     const bool lane_in = e0 < E;
     uint32_t rv[SPR];
@@ -167,33 +172,33 @@ __device__ __forceinline__ int32_t gchain_eval_cdd(const GChain<G, E>& ch, int l
     uint32_t lsum = 0;
 #pragma unroll
     for (int i = 0; i < SPR; ++i) {
-        v[i] = ((pv >> (8 * i)) & 0xffu) | (((rv[i] & 0xffffu) + (rv[i] >> 16)) << 16);
+        // p | (alpha + beta) << 16 from the widened record alpha | beta << 16
+        v[i] = __byte_perm(pv, 0u, 0x4440u + i) + (rv[i] << 16) + (rv[i] & 0xffff0000u);
         lsum += v[i];
     }
-    uint32_t ex = gscan<G>(lsum) - lsum;
-    int32_t Cex[SPR], Sex[SPR], pe[SPR];
-    uint32_t cnt = 0;
-    const int kbase = Ls * E + e0;
+    const uint32_t ex = gscan<G>(lsum) - lsum;
+    // k0: the last element of the row with S_excl <= Btot (a prefix of the row); its inclusive C
+    uint32_t run = ex, cinc = 0;
+    // (run >> 16) <= thr  <=>  run <= key   (s < 2^15, so thr >= 0xffff admits every element)
+    const uint32_t key = ((uint32_t)min(thr, 0xffff) << 16) | 0xffffu;
+    const bool sat0 = lane_in && ex <= key;
 #pragma unroll
     for (int i = 0; i < SPR; ++i) {
-        Cex[i] = PbS + (int32_t)(ex & 0xffffu);
-        Sex[i] = SbS + (int32_t)(ex >> 16);
-        pe[i] = (int32_t)(v[i] & 0xffffu);
-        cnt += (lane_in && (kbase + i < n) && (Sex[i] <= Btot)) ? 1u : 0u;
-        ex += v[i];
+        const bool sat = run <= key;
+        run += v[i];
+        cinc = sat ? run : cinc;
     }
-    const int ik = (int)gsum<G>(cnt) - 1;  // k0 - Ls*E when Ls == Lk
-    const int own = ik < 0 ? 0 : ik / SPR, ei = ik < 0 ? 0 : ik % SPR;
-    int32_t csel = Cex[0] + pe[0];
-#pragma unroll
-    for (int i = 1; i < SPR; ++i) csel = (ei == i) ? Cex[i] + pe[i] : csel;
-    const int32_t Ck0 = __shfl_sync(kFull, csel, own, G);
-    const int32_t D = (Ls == Lk) ? min(Ck0, d) : d;
+    const int own = hibit(group_ballot<G>(sat0, gbase));  // >= 0: element 0 of the row has S = SbS
+    const int32_t Ck0 = PbS + (int32_t)(__shfl_sync(kFull, cinc, own < 0 ? 0 : own, G) & 0xffffu);
+    const int32_t Dr = ((Ls == Lk) ? min(Ck0, d) : d) - PbS;  // D - C at the row start
     int32_t corr = 0;
+    run = ex;
 #pragma unroll
     for (int i = 0; i < SPR; ++i) {
-        const bool vi = lane_in && (kbase + i < n);
-        corr += vi ? (Sex[i] - Btot) * min(pe[i], max(0, D - Cex[i])) : 0;
+        const int32_t ci = (int32_t)(run & 0xffffu), si = (int32_t)(run >> 16);
+        const int32_t pi = (int32_t)(v[i] & 0xffu);
+        corr += (si - thr) * min(pi, max(0, Dr - ci));
+        run += v[i];
     }
 
     // ---- F(C_{m'}): per pair, f2 = (s, s + x0) by PRMT + IMAD, IDP.2A with the pair of p bytes,
@@ -269,25 +274,19 @@ __device__ __forceinline__ int32_t gchain_eval_ucddcp(const GChain<G, E, true>& 
 #pragma unroll
     for (int i = 0; i < SPR; ++i) lsum += rv[i];
     uint32_t ex = gscan<G>(lsum) - lsum;
-    int32_t wA[SPR], wB[SPR];
-    uint32_t cnt = 0;
-    const int kbase = Lk * E + e0;
-#pragma unroll
-    for (int i = 0; i < SPR; ++i) {
-        const int32_t Aex = (int32_t)(ABbS & 0xffffu) + (int32_t)(ex & 0xffffu);
-        const int32_t Bex = (int32_t)(ABbS >> 16) + (int32_t)(ex >> 16);
-        wA[i] = Aex;
-        wB[i] = Btot - Bex;
-        cnt += (lane_in && kbase + i < n && Aex + Bex <= Btot) ? 1u : 0u;
-        ex += rv[i];
-    }
-    const int ik = (int)gsum<G>(cnt) - 1;  // k0 - Lk*E
+    // The elements at or before k0 are those with A_excl + B_excl <= Btot (a prefix of the row);
+    // each of them switches from the tardy weight wB to the early weight wA.  Padded positions
+    // have M = X = 0 and add nothing, so no index test.
     int32_t corr = 0;
 #pragma unroll
     for (int i = 0; i < SPR; ++i) {
+        const int32_t wA = (int32_t)(ABbS & 0xffffu) + (int32_t)(ex & 0xffffu);
+        const int32_t Bex = (int32_t)(ABbS >> 16) + (int32_t)(ex >> 16);
+        const int32_t wB = Btot - Bex;
         const int32_t g = (int32_t)gv[i];
-        if (lane_in && e0 + i <= ik)
-            corr += (int32_t)mv[i] * (wA[i] - wB[i]) + (int32_t)xv[i] * (min(wA[i], g) - min(wB[i], g));
+        const int32_t c = (int32_t)mv[i] * (wA - wB) + (int32_t)xv[i] * (min(wA, g) - min(wB, g));
+        corr += (wA + Bex <= Btot) ? c : 0;
+        ex += rv[i];
     }
 
     // pass 2: pairs of weights as 16-bit halves, w2 = base2 +- f2

@@ -163,3 +163,41 @@ def test_large_chain_count_best_matches_oracle_chain(lib):
     p = oracle.sa_params(chains=1, steps=60, seed=5)
     for c in [0, 1, 4095, 4096, 12345, 19999, gid]:
         assert oracle.sa_chain(pr, p, T0, c)["E_best"] == cb[c], c
+
+
+# Edge cases (within the ABI's packed-record limits, cdd.h) of the group kernel's boundary search (one case per rows-per-lane size E = 8..64):
+# sum p > 2^16 (row-relative packing), zero penalties (every alpha 0: k0 = n; every beta 0),
+# Btot near the 2^16 limit of the ABI, d = 0 and d >= sum p.
+EDGE = [
+    (70, dict(p=(1, 255), alpha=(0, 15), beta=(0, 15), h=0.5)),
+    (150, dict(p=(1, 4), alpha=(0, 0), beta=(1, 9), h=0.3)),
+    (150, dict(p=(1, 9), alpha=(1, 9), beta=(0, 0), h=0.6)),
+    (400, dict(p=(1, 4), alpha=(100, 127), beta=(100, 127), h=0.4)),
+    (700, dict(p=(1, 255), alpha=(0, 15), beta=(0, 15), h=0.2)),
+    (700, dict(p=(1, 20), alpha=(1, 10), beta=(1, 15), h=0.0)),
+    (1000, dict(p=(1, 20), alpha=(1, 10), beta=(1, 15), h=1.2)),
+    (1000, dict(p=(1, 3), alpha=(40, 60), beta=(40, 60), h=0.45)),
+]
+
+
+@pytest.mark.parametrize("n,kw", EDGE)
+@pytest.mark.parametrize("problem", ["cdd", "ucddcp"])
+def test_edge_instances_trace_parity(lib, n, kw, problem):
+    if problem == "ucddcp" and kw["alpha"][1] == 0:
+        pytest.skip("UCDDCP gamma range needs alpha > 0")
+    inst = gen.ranged_instance(n, 9, problem=problem, **kw)
+    chains = 24
+    if problem == "ucddcp" and not lib.Instance.from_gen(inst).query()["has_ucddcp"]:
+        # M, P-M, gamma do not fit the packed UCDDCP record: refused, the CDD side still works
+        with pytest.raises(lib.CddError):
+            lib.sa_run(lib.Instance.from_gen(inst), 4, 10, problem="ucddcp", T0=1.0)
+        return
+    ins, res, (pen, perm, gid), pr, p, T0 = _run_both(lib, inst, problem, chains, 120, 31 + n,
+                                                     samples=200)
+    tr = res["trace"].cpu().numpy()
+    for c in range(chains):
+        ref = oracle.sa_chain(pr, p, T0, c, trace=True)
+        assert np.array_equal(tr[c] >> 1, ref["E_new"]), c
+        assert np.array_equal((tr[c] & 1).astype(bool), ref["accepted"]), c
+    full = oracle.sa_run(pr, p, T0)
+    assert (pen, gid) == (full["E_best"], full["g"]) and np.array_equal(perm, full["best"])
