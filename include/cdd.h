@@ -30,7 +30,7 @@
 extern "C" {
 #endif
 
-#define CDD_ABI_VERSION 1
+#define CDD_ABI_VERSION 2
 
 #if defined(__GNUC__)
 #define CDD_API __attribute__((visibility("default")))
@@ -103,7 +103,7 @@ CDD_API int cdd_check(cdd_instance *inst, void *stream);
 /* ------------------------------------------------------------------------------------------ */
 typedef struct {
     cdd_problem problem;
-    int64_t chains;        /* chains on this device (one warp each)                            */
+    int64_t chains;        /* chains on this device                                            */
     int64_t steps;         /* Alg. 1 #Iterations (1000 / 5000)                       */
     double mu;             /* exponential cooling factor (0.88)                          */
     double T0;             /* > 0: initial temperature; <= 0: T0 = std of t0_samples random    */
@@ -120,6 +120,10 @@ typedef struct {
     double *T0_out;        /* optional device double [1]: the T0 used                            */
     const double *T0_in;   /* optional device double [1]: T0 read on the device (e.g. from sa_t0); */
                            /* overrides T0 / t0_samples when non-NULL                             */
+    int32_t lanes;         /* threads per chain: 0 = automatic (by n and chains), 32 = one warp  */
+                           /* per chain, 4 / 8 / 16 = 8 / 4 / 2 chains per warp (16-bit records: */
+                           /* needs alpha, beta <= 255, else CDD_EINVAL); results do not depend  */
+                           /* on it (bit-identical), only the speed does                          */
 } sa_params;
 
 /* Bytes of device workspace sa_run needs for these parameters (caller allocates, e.g. torch). */

@@ -42,7 +42,8 @@ class SaParams(C.Structure):
                 ("mu", C.c_double), ("T0", C.c_double), ("t0_samples", C.c_int64),
                 ("pert", C.c_int32), ("move", C.c_int), ("seed", C.c_uint64),
                 ("chain_offset", C.c_uint64), ("trace", C.c_void_p), ("chain_best", C.c_void_p),
-                ("chain_final", C.c_void_p), ("T0_out", C.c_void_p), ("T0_in", C.c_void_p)]
+                ("chain_final", C.c_void_p), ("T0_out", C.c_void_p), ("T0_in", C.c_void_p),
+                ("lanes", C.c_int32)]
 
 
 class DpsoParams(C.Structure):
@@ -204,11 +205,11 @@ def cdd_check(inst: Instance, stream=None) -> None:
 
 
 def _sa_params(problem, chains, steps, mu, T0, t0_samples, pert, move, seed, chain_offset,
-               trace=None, chain_best=None, chain_final=None, T0_out=None, T0_in=None):
+               trace=None, chain_best=None, chain_final=None, T0_out=None, T0_in=None, lanes=0):
     return SaParams(PROBLEMS[problem], int(chains), int(steps), float(mu), float(T0),
                     int(t0_samples), int(pert), MOVES[move], int(seed) & (2**64 - 1),
                     int(chain_offset), _dptr(trace), _dptr(chain_best), _dptr(chain_final),
-                    _dptr(T0_out), _dptr(T0_in))
+                    _dptr(T0_out), _dptr(T0_in), int(lanes))
 
 
 def sa_workspace_size(inst: Instance, **kw) -> int:
@@ -218,10 +219,11 @@ def sa_workspace_size(inst: Instance, **kw) -> int:
 
 def sa_run(inst: Instance, chains: int, steps: int, problem="cdd", mu=0.88, T0=0.0,
            t0_samples=5000, pert=4, move="pert_fy", seed=0, chain_offset=0, trace=False,
-           chain_best=False, chain_final=False, stream=None, workspace=None, T0_dev=None):
+           chain_best=False, chain_final=False, stream=None, workspace=None, T0_dev=None, lanes=0):
     """Asynchronous parallel SA (Alg. 1): `chains` independent chains of `steps` iterations,
     reduced to the best (penalty, chain) into the instance's best buffers.  Returns the optional
-    per-chain device tensors (and the T0 used) without synchronising."""
+    per-chain device tensors (and the T0 used) without synchronising.  `lanes`: threads per
+    chain (0 automatic, 32, 16, 8, 4) -- a speed knob only, results are identical."""
     import torch
 
     dev = torch.device("cuda", inst.device)
@@ -234,7 +236,7 @@ def sa_run(inst: Instance, chains: int, steps: int, problem="cdd", mu=0.88, T0=0
         res["chain_final"] = torch.empty(chains, dtype=torch.int64, device=dev)
     p = _sa_params(problem, chains, steps, mu, T0, t0_samples, pert, move, seed, chain_offset,
                    res.get("trace"), res.get("chain_best"), res.get("chain_final"), res["T0"],
-                   T0_dev)
+                   T0_dev, lanes)
     need = int(_lib.sa_workspace_size(inst.handle, C.byref(p)))
     if need == 0:
         _check(_lib.sa_run(inst.handle, C.byref(p), None, 0, None))  # raises with the reason

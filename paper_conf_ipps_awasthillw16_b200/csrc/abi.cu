@@ -324,7 +324,13 @@ static int sa_validate(const cdd_instance* I, const sa_params* p, cdd::SaLaunch*
     if (!std::isfinite(p->mu) || p->mu < 0) return fail(CDD_EINVAL, "mu must be finite and >= 0");
     if (!(p->T0 > 0) && !p->T0_in && p->t0_samples < 1) return fail(CDD_EINVAL, "T0 <= 0 needs t0_samples >= 1");
     if (std::isnan(p->T0)) return fail(CDD_EINVAL, "T0 is NaN");
+    if (p->lanes != 0 && p->lanes != 4 && p->lanes != 8 && p->lanes != 16 && p->lanes != 32)
+        return fail(CDD_EINVAL, "lanes must be 0, 4, 8, 16 or 32");
+    if (p->lanes >= 4 && p->lanes <= 16 && !I->ab16_ok)
+        return fail(CDD_EINVAL, "lanes 4/8/16 need alpha, beta <= 255 (16-bit records)");
+    if (p->lanes == 4 && I->n > 256) return fail(CDD_EINVAL, "lanes = 4 supports n <= 256");
     L->ucd = ucd;
+    L->lanes = p->lanes;
     L->chains = p->chains;
     L->steps = p->steps;
     L->mu = p->mu;

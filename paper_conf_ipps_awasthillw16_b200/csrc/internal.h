@@ -64,6 +64,7 @@ struct SaLaunch {
     int64_t *trace, *chain_best, *chain_final;
     double* T0_out;
     const double* T0_in;
+    int32_t lanes;  // 0 automatic, 32 warp per chain, 4 / 8 / 16 group kernel
 };
 size_t sa_workspace_bytes(const Instance& I, const SaLaunch& p);
 cudaError_t launch_t0(const Instance& I, bool ucd, uint64_t seed, int64_t samples, double* T0_dev,

@@ -37,7 +37,7 @@ template <int G, int E, bool UCD = false>
 struct GChain {
     static constexpr int NP = G * E;
     static constexpr int AS = E >= 16 ? 2 * E + 16 : 2 * E;               // bytes per lane row (ab)
-    static constexpr int PS = E == 64 ? 80 : (E == 32 ? 48 : E);            // bytes per lane row (p)
+    static constexpr int PS = E >= 32 ? E + 16 : E;                        // bytes per lane row (p)
     static constexpr int GS = E >= 16 ? 2 * E + 16 : 2 * E;                // bytes per lane row (gamma)
     static constexpr int SPR = E >= G ? E / G : 1;                         // boundary elements per lane
     static constexpr int AB_BYTES = (G * AS + 15) / 16 * 16;
@@ -115,7 +115,18 @@ __device__ __forceinline__ void load_b8(const uint8_t* row, uint32_t (&w)[E / 4]
 template <int SPR, class C>
 __device__ __forceinline__ void load_spread(const C& ch, int ls, int e0, bool in, uint32_t (&rv)[SPR]) {
     const uint16_t* src = ch.ab() + ls * (C::AS / 2) + e0;
-    if constexpr (SPR == 4) {
+    if constexpr (SPR >= 8) {
+#pragma unroll
+        for (int v = 0; v < SPR / 8; ++v) {
+            const uint4 x = reinterpret_cast<const uint4*>(src)[v];
+            const uint32_t w[4] = {x.x, x.y, x.z, x.w};
+#pragma unroll
+            for (int i = 0; i < 4; ++i) {
+                rv[8 * v + 2 * i] = ab_wide(w[i] & 0xffffu);
+                rv[8 * v + 2 * i + 1] = ab_wide(w[i] >> 16);
+            }
+        }
+    } else if constexpr (SPR == 4) {
         const uint2 x = *reinterpret_cast<const uint2*>(src);
         rv[0] = ab_wide(x.x & 0xffffu); rv[1] = ab_wide(x.x >> 16);
         rv[2] = ab_wide(x.y & 0xffffu); rv[3] = ab_wide(x.y >> 16);
@@ -125,6 +136,99 @@ __device__ __forceinline__ void load_spread(const C& ch, int ls, int e0, bool in
     } else {
         rv[0] = in ? ab_wide(src[0]) : 0u;
     }
+}
+
+// Boundary row Ls for rows of E >= G^2 positions, in two levels, returning this lane's share of
+// corr = sum_k (S_k - Btot) * clamp(D - C_{k-1}, 0, p_k) over the row (row-relative: c_k, s_k
+// exclusive prefixes of p and alpha + beta, thr = Btot - S at the row start).
+//  level 1: lane l takes sub-block l (SB = E/G consecutive positions): its sums of p and
+//           alpha + beta (IDP.4A), its local dot  sum_k p_k * s^loc_k  (f2 pairs + IDP.2A), and a
+//           G-lane scan of the packed sums gives every sub-block's start.  Sub-blocks wholly left
+//           of D contribute  dot + (s_b - thr) * P_b  each.
+//  level 2: the sub-block holding k0 (last start with S <= Btot) is spread over the G lanes
+//           (SB/G positions each) to find C_{k0}, hence D; then the sub-block holding D (last start
+//           with c < D) is spread the same way for its partial term.
+template <int G, int E>
+__device__ __forceinline__ int32_t boundary_two_level(const GChain<G, E>& ch, int l, int gbase,
+                                                      int Ls, int Lk, int32_t d, int32_t PbS,
+                                                      int32_t thr, uint32_t key) {
+    using C = GChain<G, E>;
+    constexpr int SB = E / G;   // positions per sub-block (16 for E = 128, G = 8)
+    constexpr int L2 = SB / G;  // positions per lane in level 2
+    static_assert(SB % 8 == 0 && L2 >= 1 && L2 <= 4, "two-level boundary layout");
+    const uint8_t* arow = reinterpret_cast<const uint8_t*>(ch.ab()) + Ls * C::AS;
+    const uint8_t* prow = ch.pb() + Ls * C::PS;
+    // ---- level 1
+    uint32_t w[SB / 2], q[SB / 4];
+    load_ab16<SB>(arow + 2 * SB * l, w);
+    load_b8<SB>(prow + SB * l, q);
+    uint32_t Pb1 = 0, Sb1 = 0, sig2 = 0, dot = 0;
+#pragma unroll
+    for (int j = 0; j < SB / 4; ++j) Pb1 = __dp4a(q[j], 0x01010101u, Pb1);
+#pragma unroll
+    for (int j = 0; j < SB / 2; ++j) {
+        // positions 2j, 2j+1: f2 = (s, s + s_{2j}) in 16-bit halves, dotted with (p_{2j}, p_{2j+1})
+        const uint32_t f2 = __dp4a(w[j], 0x00000101u, 0u) * 0x10000u + sig2;
+        dot = (j & 1) ? __dp2a_hi(f2, q[j >> 1], dot) : __dp2a_lo(f2, q[j >> 1], dot);
+        const uint32_t pair = __dp4a(w[j], 0x01010101u, 0u);
+        sig2 += pair * 0x10001u;
+        Sb1 += pair;
+    }
+    const uint32_t lsum = Pb1 | (Sb1 << 16);
+    const uint32_t ex = gscan<G>(lsum) - lsum;  // c_b | s_b << 16 at the sub-block start
+    const int32_t cb = (int32_t)(ex & 0xffffu), sb = (int32_t)(ex >> 16);
+    const int32_t full = (int32_t)dot + (sb - thr) * (int32_t)Pb1;
+    const int own = max(0, hibit(group_ballot<G>(ex <= key, gbase)));  // lane 0 always qualifies
+
+    // ---- level 2a: k0 inside sub-block `own`, C_{k0} (inclusive) -> D
+    auto spread = [&](int blk, uint32_t (&v)[L2]) -> uint32_t {
+        const int e = SB * blk + L2 * l;
+        uint32_t a2[(L2 + 1) / 2], pp;
+        if constexpr (L2 == 4) {
+            const uint2 x = *reinterpret_cast<const uint2*>(arow + 2 * e);
+            a2[0] = x.x; a2[1] = x.y;
+            pp = *reinterpret_cast<const uint32_t*>(prow + e);
+        } else if constexpr (L2 == 2) {
+            a2[0] = *reinterpret_cast<const uint32_t*>(arow + 2 * e);
+            pp = *reinterpret_cast<const uint16_t*>(prow + e);
+        } else {
+            a2[0] = *reinterpret_cast<const uint16_t*>(arow + 2 * e);
+            pp = prow[e];
+        }
+        uint32_t tot = 0;
+#pragma unroll
+        for (int i = 0; i < L2; ++i) {
+            const uint32_t si = __dp4a(a2[i >> 1], (i & 1) ? 0x01010000u : 0x00000101u, 0u);
+            v[i] = __byte_perm(pp, 0u, 0x4440u + i) + (si << 16);
+            tot += v[i];
+        }
+        return gscan<G>(tot) - tot + __shfl_sync(kFull, ex, blk, G);  // row-relative start
+    };
+    uint32_t v[L2];
+    uint32_t run = spread(own, v), cinc = 0;
+    const bool first_sat = run <= key;
+#pragma unroll
+    for (int i = 0; i < L2; ++i) {
+        const bool sat = run <= key;
+        run += v[i];
+        cinc = sat ? run : cinc;
+    }
+    const int own2 = max(0, hibit(group_ballot<G>(first_sat, gbase)));
+    const int32_t Ck0 = PbS + (int32_t)(__shfl_sync(kFull, cinc, own2, G) & 0xffffu);
+    const int32_t Dr = ((Ls == Lk) ? min(Ck0, d) : d) - PbS;  // D - C at the row start
+
+    // ---- level 2b: sub-blocks left of the one holding D count in full; that one in part
+    const int ownD = hibit(group_ballot<G>(cb < Dr, gbase));  // -1 iff Dr <= 0 (then corr = 0)
+    run = spread(max(ownD, 0), v);
+    int32_t corr = (l < ownD) ? full : 0;
+#pragma unroll
+    for (int i = 0; i < L2; ++i) {
+        const int32_t ci = (int32_t)(run & 0xffffu), si = (int32_t)(run >> 16);
+        const int32_t pi = (int32_t)(v[i] & 0xffu);
+        corr += (si - thr) * min(pi, max(0, Dr - ci));
+        run += v[i];
+    }
+    return corr;
 }
 
 // CDD penalty of the group's chain.  tAB / tP: this lane's totals (maintained incrementally).
@@ -155,50 +259,66 @@ __device__ __forceinline__ int32_t gchain_eval_cdd(const GChain<G, E>& ch, int l
     const int32_t PbS = __shfl_sync(kFull, Pb, Ls, G);
     const uint32_t ABbS = __shfl_sync(kFull, ABb, Ls, G);
     const int32_t SbS = (int32_t)(ABbS & 0xffffu) + (int32_t)(ABbS >> 16);
-    // Everything below is relative to the start of the row: C - PbS and S - SbS, both < 2^15 per
-    // row (E * 255, E * 510), so they travel packed as c | s << 16.  thr = Btot - SbS >= 0 since
+    // Everything below is relative to the start of the row: C - PbS and S - SbS, both < 2^16 per
+    // row (E * 255, E * 510 for E <= 128), so they travel packed as c | s << 16.  thr = Btot - SbS >= 0 since
     // Ls <= Lk.  Padded positions (k >= n) hold zero records: they add nothing to c or s, and where
     // they pass the S <= Btot test (only if every alpha is 0) they repeat C_n, so no index test.
     const int32_t thr = Btot - SbS;
-    const int e0 = l * SPR;
-    const bool lane_in = e0 < E;
-    uint32_t rv[SPR];
-    load_spread<SPR>(ch, Ls, e0, lane_in, rv);
-    uint32_t pv = 0;
-    if constexpr (SPR == 4) pv = *reinterpret_cast<const uint32_t*>(ch.pb() + Ls * C::PS + e0);
-    else if constexpr (SPR == 2) pv = *reinterpret_cast<const uint16_t*>(ch.pb() + Ls * C::PS + e0);
-    else pv = lane_in ? ch.pb()[Ls * C::PS + e0] : 0u;
-    uint32_t v[SPR];
-    uint32_t lsum = 0;
-#pragma unroll
-    for (int i = 0; i < SPR; ++i) {
-        // p | (alpha + beta) << 16 from the widened record alpha | beta << 16
-        v[i] = __byte_perm(pv, 0u, 0x4440u + i) + (rv[i] << 16) + (rv[i] & 0xffff0000u);
-        lsum += v[i];
-    }
-    const uint32_t ex = gscan<G>(lsum) - lsum;
-    // k0: the last element of the row with S_excl <= Btot (a prefix of the row); its inclusive C
-    uint32_t run = ex, cinc = 0;
-    // (run >> 16) <= thr  <=>  run <= key   (s < 2^15, so thr >= 0xffff admits every element)
+    // (s >> 16) <= thr  <=>  s <= key  for a packed c | s << 16 (s <= E * 510 < 2^16, so
+    // thr >= 0xffff admits every element)
     const uint32_t key = ((uint32_t)min(thr, 0xffff) << 16) | 0xffffu;
-    const bool sat0 = lane_in && ex <= key;
-#pragma unroll
-    for (int i = 0; i < SPR; ++i) {
-        const bool sat = run <= key;
-        run += v[i];
-        cinc = sat ? run : cinc;
-    }
-    const int own = hibit(group_ballot<G>(sat0, gbase));  // >= 0: element 0 of the row has S = SbS
-    const int32_t Ck0 = PbS + (int32_t)(__shfl_sync(kFull, cinc, own < 0 ? 0 : own, G) & 0xffffu);
-    const int32_t Dr = ((Ls == Lk) ? min(Ck0, d) : d) - PbS;  // D - C at the row start
     int32_t corr = 0;
-    run = ex;
+    if constexpr (E < G * G || E / G < 8) {  // one level: SPR = E/G positions per lane
+        const int e0 = l * SPR;
+        const bool lane_in = e0 < E;
+        uint32_t rv[SPR];
+        load_spread<SPR>(ch, Ls, e0, lane_in, rv);
+        constexpr int PW = SPR >= 4 ? SPR / 4 : 1;
+        uint32_t pv[PW];
+        const uint8_t* psrc = ch.pb() + Ls * C::PS + e0;
+        if constexpr (SPR >= 16) {
 #pragma unroll
-    for (int i = 0; i < SPR; ++i) {
-        const int32_t ci = (int32_t)(run & 0xffffu), si = (int32_t)(run >> 16);
-        const int32_t pi = (int32_t)(v[i] & 0xffu);
-        corr += (si - thr) * min(pi, max(0, Dr - ci));
-        run += v[i];
+            for (int q = 0; q < SPR / 16; ++q) {
+                const uint4 x = reinterpret_cast<const uint4*>(psrc)[q];
+                pv[4 * q] = x.x; pv[4 * q + 1] = x.y; pv[4 * q + 2] = x.z; pv[4 * q + 3] = x.w;
+            }
+        } else if constexpr (SPR == 8) {
+            const uint2 x = *reinterpret_cast<const uint2*>(psrc);
+            pv[0] = x.x; pv[1] = x.y;
+        } else if constexpr (SPR == 4) pv[0] = *reinterpret_cast<const uint32_t*>(psrc);
+        else if constexpr (SPR == 2) pv[0] = *reinterpret_cast<const uint16_t*>(psrc);
+        else pv[0] = lane_in ? psrc[0] : 0u;
+        uint32_t v[SPR];
+        uint32_t lsum = 0;
+#pragma unroll
+        for (int i = 0; i < SPR; ++i) {
+            // p | (alpha + beta) << 16 from the widened record alpha | beta << 16
+            v[i] = __byte_perm(pv[i / 4], 0u, 0x4440u + (i & 3)) + (rv[i] << 16) + (rv[i] & 0xffff0000u);
+            lsum += v[i];
+        }
+        const uint32_t ex = gscan<G>(lsum) - lsum;
+        // k0: the last element of the row with S_excl <= Btot (a prefix of the row); its inclusive C
+        uint32_t run = ex, cinc = 0;
+        const bool sat0 = lane_in && ex <= key;
+#pragma unroll
+        for (int i = 0; i < SPR; ++i) {
+            const bool sat = run <= key;
+            run += v[i];
+            cinc = sat ? run : cinc;
+        }
+        const int own = hibit(group_ballot<G>(sat0, gbase));  // >= 0: element 0 of the row has S = SbS
+        const int32_t Ck0 = PbS + (int32_t)(__shfl_sync(kFull, cinc, own < 0 ? 0 : own, G) & 0xffffu);
+        const int32_t Dr = ((Ls == Lk) ? min(Ck0, d) : d) - PbS;  // D - C at the row start
+        run = ex;
+#pragma unroll
+        for (int i = 0; i < SPR; ++i) {
+            const int32_t ci = (int32_t)(run & 0xffffu), si = (int32_t)(run >> 16);
+            const int32_t pi = (int32_t)(v[i] & 0xffu);
+            corr += (si - thr) * min(pi, max(0, Dr - ci));
+            run += v[i];
+        }
+    } else {
+        corr = boundary_two_level<G, E>(ch, l, gbase, Ls, Lk, d, PbS, thr, key);
     }
 
     // ---- F(C_{m'}): per pair, f2 = (s, s + x0) by PRMT + IMAD, IDP.2A with the pair of p bytes,

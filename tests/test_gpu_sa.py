@@ -34,14 +34,22 @@ def test_t0_bit_exact(lib, n, problem):
     assert t_gpu == t_ref  # same double, bit for bit
 
 
+# threads per chain: 32 = warp kernel, 16 / 8 / 4 = group kernel (2 / 4 / 8 chains per warp)
+LANES = [32, 16, 8, 4]
+
+
+def _lanes_ok(n, lanes):
+    return lanes != 4 or n <= 256
+
+
 def _run_both(lib, inst, problem, chains, steps, seed, T0=0.0, samples=5000, move="pert_fy",
-              pert=4, chain_offset=0, trace=True, mu=0.88):
+              pert=4, chain_offset=0, trace=True, mu=0.88, lanes=0):
     import torch
 
     ins = lib.Instance.from_gen(inst)
     res = lib.sa_run(ins, chains, steps, problem=problem, mu=mu, T0=T0, t0_samples=samples,
                      pert=pert, move=move, seed=seed, chain_offset=chain_offset, trace=trace,
-                     chain_best=True, chain_final=True)
+                     chain_best=True, chain_final=True, lanes=lanes)
     torch.cuda.synchronize()
     pen, perm, gid = lib.best_get(ins)
     pr = _prob(inst)
@@ -67,13 +75,16 @@ def test_config1_single_chain_10k_steps_trace(lib):
     assert int(res["chain_final"].item()) == ref["E_final"]
 
 
+@pytest.mark.parametrize("lanes", LANES)
 @pytest.mark.parametrize("n,chains,steps", [(4, 40, 300), (17, 64, 400), (100, 256, 2000),
-                                            (250, 96, 500), (1000, 32, 300)])
-def test_many_chains_trace_parity(lib, n, chains, steps):
+                                            (250, 96, 500), (600, 40, 300), (1000, 32, 300)])
+def test_many_chains_trace_parity(lib, n, chains, steps, lanes):
+    if not _lanes_ok(n, lanes):
+        pytest.skip("lanes=4 needs n <= 256")
     inst = gen.cdd_instance(n, 2, 0.6)
     seed = 1000 + n
     ins, res, (pen, perm, gid), pr, p, T0 = _run_both(lib, inst, "cdd", chains, steps, seed,
-                                                     samples=800)
+                                                     samples=800, lanes=lanes)
     tr = res["trace"].cpu().numpy()
     cb = res["chain_best"].cpu().numpy()
     cf = res["chain_final"].cpu().numpy()
@@ -87,12 +98,15 @@ def test_many_chains_trace_parity(lib, n, chains, steps):
     assert np.array_equal(perm, full["best"])
 
 
+@pytest.mark.parametrize("lanes", LANES)
 @pytest.mark.parametrize("n,chains,steps", [(40, 32, 300), (200, 48, 400), (333, 40, 200),
                                             (1000, 20, 150)])
-def test_ucddcp_sa_parity(lib, n, chains, steps):
+def test_ucddcp_sa_parity(lib, n, chains, steps, lanes):
+    if not _lanes_ok(n, lanes):
+        pytest.skip("lanes=4 needs n <= 256")
     inst = gen.ucddcp_instance(n, 4)
     ins, res, (pen, perm, gid), pr, p, T0 = _run_both(lib, inst, "ucddcp", chains, steps, 77,
-                                                     samples=600)
+                                                     samples=600, lanes=lanes)
     cb = res["chain_best"].cpu().numpy()
     tr = res["trace"].cpu().numpy()
     for c in range(chains):
@@ -103,11 +117,12 @@ def test_ucddcp_sa_parity(lib, n, chains, steps):
     assert oracle.ucddcp_eval(pr, perm) == pen
 
 
+@pytest.mark.parametrize("lanes", [32, 8, 4])
 @pytest.mark.parametrize("move,pert", [("swap", 4), ("pert_fy", 2), ("pert_fy", 3), ("pert_fy", 1)])
-def test_move_variants(lib, move, pert):
+def test_move_variants(lib, move, pert, lanes):
     inst = gen.cdd_instance(60, 5, 0.2)
     ins, res, (pen, perm, gid), pr, p, T0 = _run_both(lib, inst, "cdd", 32, 300, 5, move=move,
-                                                     pert=pert, samples=300)
+                                                     pert=pert, samples=300, lanes=lanes)
     tr = res["trace"].cpu().numpy()
     for c in range(32):
         ref = oracle.sa_chain(pr, p, T0, c, trace=True)
@@ -180,11 +195,14 @@ EDGE = [
 ]
 
 
+@pytest.mark.parametrize("lanes", [0] + LANES)
 @pytest.mark.parametrize("n,kw", EDGE)
 @pytest.mark.parametrize("problem", ["cdd", "ucddcp"])
-def test_edge_instances_trace_parity(lib, n, kw, problem):
+def test_edge_instances_trace_parity(lib, n, kw, problem, lanes):
     if problem == "ucddcp" and kw["alpha"][1] == 0:
         pytest.skip("UCDDCP gamma range needs alpha > 0")
+    if not _lanes_ok(n, lanes):
+        pytest.skip("lanes=4 needs n <= 256")
     inst = gen.ranged_instance(n, 9, problem=problem, **kw)
     chains = 24
     if problem == "ucddcp" and not lib.Instance.from_gen(inst).query()["has_ucddcp"]:
@@ -193,7 +211,7 @@ def test_edge_instances_trace_parity(lib, n, kw, problem):
             lib.sa_run(lib.Instance.from_gen(inst), 4, 10, problem="ucddcp", T0=1.0)
         return
     ins, res, (pen, perm, gid), pr, p, T0 = _run_both(lib, inst, problem, chains, 120, 31 + n,
-                                                     samples=200)
+                                                     samples=200, lanes=lanes)
     tr = res["trace"].cpu().numpy()
     for c in range(chains):
         ref = oracle.sa_chain(pr, p, T0, c, trace=True)
@@ -201,3 +219,20 @@ def test_edge_instances_trace_parity(lib, n, kw, problem):
         assert np.array_equal((tr[c] & 1).astype(bool), ref["accepted"]), c
     full = oracle.sa_run(pr, p, T0)
     assert (pen, gid) == (full["E_best"], full["g"]) and np.array_equal(perm, full["best"])
+
+
+def test_lanes_argument_checks(lib):
+    big = gen.cdd_instance(300, 1, 0.4)
+    with pytest.raises(lib.CddError):
+        lib.sa_run(lib.Instance.from_gen(big), 64, 10, T0=5.0, lanes=4)  # n > 256
+    with pytest.raises(lib.CddError):
+        lib.sa_run(lib.Instance.from_gen(big), 64, 10, T0=5.0, lanes=12)
+    # alpha > 255: no 16-bit records, the group layouts refuse, the warp layout runs
+    heavy = gen.ranged_instance(80, 3, p=(1, 3), alpha=(200, 400), beta=(1, 5), h=0.5)
+    ins = lib.Instance.from_gen(heavy)
+    with pytest.raises(lib.CddError):
+        lib.sa_run(ins, 64, 10, T0=5.0, lanes=8)
+    lib.sa_run(ins, 64, 10, T0=5.0, lanes=32)
+    lib.sa_run(ins, 4096, 10, T0=5.0)  # automatic: warp layout
+    pen, perm, gid = lib.best_get(ins)
+    assert oracle.cdd_eval(_prob(heavy), perm) == pen
