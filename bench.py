@@ -289,8 +289,11 @@ def main():
     if os.path.exists(tp):
         traffic = json.load(open(tp)).get("dram_bytes_per_launch")
     step_ms = ms / args.steps
+    G, E = lib.sa_layout(insts[0], chains)
+    kname = (f"sa_group_kernel<{G},{E}> (CDD, {32 // G} chains per warp)" if G < 32
+             else f"sa_kernel<{E}> (CDD, one warp per chain)")
     roofline = {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "Tint-op/s",
-                "frac": achieved / peak, "traffic": traffic, "kernel": "sa_group_kernel<16,64> (CDD, 2 chains per warp)",
+                "frac": achieved / peak, "traffic": traffic, "kernel": kname,
                 "kernel_ms_avg": k_avg_ms, "kernel_share_of_step": k_avg_ms * len(insts) / step_ms,
                 "ops_per_launch": ops,
                 "peak_note": f"128 int32 lane-ops/clk/SM (4 SMSP x 32 lanes issue, alu+fma pipes) x {nsm} SMs x {sm_max:.0f} MHz max clock"}

@@ -132,6 +132,11 @@ CDD_API size_t sa_workspace_size(const cdd_instance *inst, const sa_params *para
  * reduces min (best penalty, global chain id) into the instance's best buffers. */
 CDD_API int sa_run(cdd_instance *inst, const sa_params *params, void *workspace, size_t workspace_bytes,
            void *stream);
+/* The thread layout sa_run would use for these parameters: *lanes threads per chain (32: one
+ * warp per chain; 4 / 8 / 16: 8 / 4 / 2 chains per warp) holding *positions_per_lane sequence
+ * positions each (lanes x positions >= n).  Host-only, synchronous; either out may be NULL. */
+CDD_API int sa_layout(const cdd_instance *inst, const sa_params *params, int32_t *lanes,
+                      int32_t *positions_per_lane);
 /* ASYNC.  Only the T0 rule: *T0_dev = population std of the penalties of `samples`
  * Philox-random sequences.  Workspace: sa_workspace_size() of an sa_params with T0 <= 0. */
 CDD_API int sa_t0(cdd_instance *inst, cdd_problem problem, uint64_t seed, int64_t samples, double *T0_dev,

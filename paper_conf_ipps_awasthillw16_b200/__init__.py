@@ -64,6 +64,7 @@ _SIGS = {
     "sa_workspace_size": (_sz, [_vp, C.POINTER(SaParams)]),
     "sa_run": (C.c_int, [_vp, C.POINTER(SaParams), _vp, _sz, _vp]),
     "sa_t0": (C.c_int, [_vp, C.c_int, _u64, _i64, _vp, _vp, _sz, _vp]),
+    "sa_layout": (C.c_int, [_vp, C.POINTER(SaParams), _vp, _vp]),
     "dpso_workspace_size": (_sz, [_vp, C.POINTER(DpsoParams)]),
     "dpso_run": (C.c_int, [_vp, C.POINTER(DpsoParams), _vp, _sz, _vp]),
     "dpso_begin": (C.c_int, [_vp, C.POINTER(DpsoParams), _vp, _sz, _vp]),
@@ -245,6 +246,14 @@ def sa_run(inst: Instance, chains: int, steps: int, problem="cdd", mu=0.88, T0=0
     res["workspace"] = workspace
     _check(_lib.sa_run(inst.handle, C.byref(p), workspace.data_ptr(), need, _stream(stream)))
     return res
+
+
+def sa_layout(inst: Instance, chains: int, problem="cdd", lanes=0):
+    """(threads per chain, positions per thread) that sa_run uses for these arguments."""
+    p = _sa_params(problem, chains, 1, 0.88, 1.0, 0, 4, "pert_fy", 0, 0, lanes=lanes)
+    g, e = C.c_int32(), C.c_int32()
+    _check(_lib.sa_layout(inst.handle, C.byref(p), C.byref(g), C.byref(e)))
+    return g.value, e.value
 
 
 def sa_t0(inst: Instance, problem="cdd", seed=0, samples=5000, stream=None):

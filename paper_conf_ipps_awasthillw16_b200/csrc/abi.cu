@@ -355,6 +355,17 @@ size_t sa_workspace_size(const cdd_instance* I, const sa_params* p) {
     return cdd::sa_workspace_bytes(*I, L);
 }
 
+int sa_layout(const cdd_instance* I, const sa_params* p, int32_t* lanes, int32_t* positions_per_lane) {
+    cdd::SaLaunch L{};
+    const int rc = sa_validate(I, p, &L);
+    if (rc != CDD_OK) return rc;
+    int32_t g = 0, e = 0;
+    cdd::sa_layout(*I, L, &g, &e);
+    if (lanes) *lanes = g;
+    if (positions_per_lane) *positions_per_lane = e;
+    return CDD_OK;
+}
+
 int sa_run(cdd_instance* I, const sa_params* p, void* ws, size_t ws_bytes, void* stream) {
     cdd::SaLaunch L{};
     int rc = sa_validate(I, p, &L);

@@ -70,6 +70,7 @@ size_t sa_workspace_bytes(const Instance& I, const SaLaunch& p);
 cudaError_t launch_t0(const Instance& I, bool ucd, uint64_t seed, int64_t samples, double* T0_dev,
                       void* ws, cudaStream_t s);
 cudaError_t launch_sa(Instance& I, const SaLaunch& p, void* ws, cudaStream_t s);
+void sa_layout(const Instance& I, const SaLaunch& p, int32_t* lanes, int32_t* per_lane);
 
 // ---- launchers (dpso.cu) ----
 struct DpsoLaunch {

@@ -236,3 +236,13 @@ def test_lanes_argument_checks(lib):
     lib.sa_run(ins, 4096, 10, T0=5.0)  # automatic: warp layout
     pen, perm, gid = lib.best_get(ins)
     assert oracle.cdd_eval(_prob(heavy), perm) == pen
+
+
+def test_sa_layout_query(lib):
+    for n, chains, lanes in [(1000, 65536, 0), (100, 16384, 0), (100, 100, 0), (300, 4096, 16),
+                             (50, 8192, 4), (700, 2048, 32)]:
+        ins = lib.Instance.from_gen(gen.cdd_instance(n, 1, 0.4))
+        g, e = lib.sa_layout(ins, chains, lanes=lanes)
+        assert g in (4, 8, 16, 32) and g * e >= n and (lanes == 0 or g == lanes)
+        if chains < 1024:
+            assert g == 32
