@@ -4,9 +4,9 @@ set -x
 mkdir -p gpurun_out
 python bench.py --steps 3 --warmup 3 > gpurun_out/bench_full.json 2> gpurun_out/bench_full.err
 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches.csv \
-    python bench.py --steps 1 --warmup 0 --no-cpu-baseline --no-e2e --no-eval > /dev/null 2>&1
+    python bench.py --steps 1 --warmup 0 --no-cpu-baseline --no-e2e --no-eval --no-configs > /dev/null 2>&1
 ncu --set full --clock-control none --import-source on -k regex:sa_group -c 1 -o gpurun_out/prof_sa_full \
-    python bench.py --steps 1 --warmup 0 --no-cpu-baseline --no-e2e --no-eval > /dev/null 2>&1
+    python bench.py --steps 1 --warmup 0 --no-cpu-baseline --no-e2e --no-eval --no-configs > /dev/null 2>&1
 ncu --set full --clock-control none --import-source on -k regex:eval_batch -s 3 -c 1 -o gpurun_out/prof_eval_full \
     python bench.py --steps 1 --warmup 0 --sa-steps 10 --chains 1024 --no-cpu-baseline --no-e2e > /dev/null 2>&1
 ls -la gpurun_out
