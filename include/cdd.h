@@ -94,6 +94,20 @@ CDD_API int ucddcp_eval_batch(cdd_instance *inst, const int16_t *perms, int64_t 
  * device in chunks, evaluates, copies the penalties to out_host (int64 [batch]), synchronises. */
 CDD_API int cdd_eval_batch_host(cdd_instance *inst, cdd_problem problem, const int16_t *perms_host,
                         int64_t ld, int64_t batch, int64_t *out_host, void *stream);
+/* ASYNC.  The optimal schedule of each row (what the O(n) routine finds: P:94-122 for the CDD,
+ * P:137-166 for the UCDDCP), for inspection or for materialising the best sequence of a run.
+ *   C       device int64 [batch][n]: completion time of the job at each position;
+ *   X       device int32 [batch][n]: UCDDCP compressions (NULL for the CDD);
+ *   start   device int64 [batch]: start time of the first job;
+ *   penalty device int64 [batch]: eq. (1) / (2) of this schedule, equal to the *_eval_batch value.
+ * With k0 = max{k : S_k <= sum beta} (S_k = sum of alpha + beta before position k), job k0 completes
+ * at d when C_{k0} <= d, else the schedule starts at 0 (CDD); UCDDCP: job k0 completes at d and job
+ * k is compressed fully iff its weight (A_{k-1} for k <= k0, else B_k) exceeds gamma_k.  When the
+ * cost has a flat optimum the schedule is one of the optimal ones (the penalty is unique).  Ids
+ * outside [0, n) raise the data-error flag as in cdd_eval_batch. */
+CDD_API int cdd_schedule_batch(cdd_instance *inst, cdd_problem problem, const int16_t *perms,
+                               int64_t ld, int64_t batch, int64_t *C, int32_t *X, int64_t *start,
+                               int64_t *penalty, void *stream);
 /* Synchronises `stream`; returns CDD_EDATA (and clears the flag) if any evaluated sequence held
  * a job id outside [0, n) since the last check, else CDD_OK. */
 CDD_API int cdd_check(cdd_instance *inst, void *stream);

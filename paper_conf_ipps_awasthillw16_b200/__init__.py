@@ -61,6 +61,7 @@ _SIGS = {
     "ucddcp_eval_batch": (C.c_int, [_vp, _vp, _i64, _i64, _vp, _vp]),
     "cdd_eval_batch_host": (C.c_int, [_vp, C.c_int, _vp, _i64, _i64, _vp, _vp]),
     "cdd_check": (C.c_int, [_vp, _vp]),
+    "cdd_schedule_batch": (C.c_int, [_vp, C.c_int, _vp, _i64, _i64, _vp, _vp, _vp, _vp, _vp]),
     "sa_workspace_size": (_sz, [_vp, C.POINTER(SaParams)]),
     "sa_run": (C.c_int, [_vp, C.POINTER(SaParams), _vp, _sz, _vp]),
     "sa_t0": (C.c_int, [_vp, C.c_int, _u64, _i64, _vp, _vp, _sz, _vp]),
@@ -182,6 +183,39 @@ def cdd_eval_batch(inst: Instance, perms, out=None, stream=None):
 def ucddcp_eval_batch(inst: Instance, perms, out=None, stream=None):
     """out[b] = optimal UCDDCP penalty of sequence perms[b, :n]."""
     return _eval(_lib.ucddcp_eval_batch, inst, perms, out, stream)
+
+
+def cdd_schedule_batch(inst: Instance, perms, problem="cdd", stream=None):
+    """Optimal schedules of device int16 [B, ld] sequences: dict of device tensors C [B, n] (int64),
+    X [B, n] (int32, UCDDCP), start [B], penalty [B]."""
+    import torch
+
+    assert perms.dtype == torch.int16 and perms.dim() == 2 and perms.is_cuda and perms.stride(1) == 1
+    B, ld = perms.shape[0], perms.stride(0)
+    dev = perms.device
+    out = {"C": torch.empty((B, inst.n), dtype=torch.int64, device=dev),
+           "start": torch.empty(B, dtype=torch.int64, device=dev),
+           "penalty": torch.empty(B, dtype=torch.int64, device=dev)}
+    if problem == "ucddcp":
+        out["X"] = torch.empty((B, inst.n), dtype=torch.int32, device=dev)
+    _check(_lib.cdd_schedule_batch(inst.handle, PROBLEMS[problem], perms.data_ptr(), ld, B,
+                                   out["C"].data_ptr(), _dptr(out.get("X")), out["start"].data_ptr(),
+                                   out["penalty"].data_ptr(), _stream(stream)))
+    return out
+
+
+def schedule_get(inst: Instance, perm, problem="cdd"):
+    """Optimal schedule of one host sequence (e.g. best_get's): numpy C (int64 [n]), X (int32 [n]
+    or None), start, penalty.  Synchronous."""
+    import torch
+
+    ld = (inst.n + 7) // 8 * 8
+    p = torch.zeros((1, ld), dtype=torch.int16)
+    p[0, :inst.n] = torch.from_numpy(np.ascontiguousarray(perm, dtype=np.int16))
+    out = cdd_schedule_batch(inst, p.to(torch.device("cuda", inst.device)), problem)
+    torch.cuda.synchronize(inst.device)
+    X = out["X"][0].cpu().numpy() if "X" in out else None
+    return out["C"][0].cpu().numpy(), X, int(out["start"][0].item()), int(out["penalty"][0].item())
 
 
 def cdd_eval_batch_host(inst: Instance, perms: np.ndarray, problem="cdd", out=None, stream=None):

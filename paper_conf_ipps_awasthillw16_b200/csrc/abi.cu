@@ -261,6 +261,20 @@ int ucddcp_eval_batch(cdd_instance* I, const int16_t* perms, int64_t ld, int64_t
     return eval_common(I, true, perms, ld, batch, out, stream);
 }
 
+int cdd_schedule_batch(cdd_instance* I, cdd_problem problem, const int16_t* perms, int64_t ld,
+                       int64_t batch, int64_t* C, int32_t* X, int64_t* start, int64_t* penalty,
+                       void* stream) {
+    int rc = check_batch_args(I, perms, ld, batch, penalty);
+    if (rc != CDD_OK) return rc;
+    if (problem != CDD_PROBLEM_CDD && problem != CDD_PROBLEM_UCDDCP) return fail(CDD_EINVAL, "bad problem");
+    const bool ucd = problem == CDD_PROBLEM_UCDDCP;
+    if (batch > 0 && (!C || !start || (ucd && !X))) return fail(CDD_EINVAL, "C/start (and X for UCDDCP) must be non-NULL");
+    if (ucd && (!I->has_ucd || I->d < I->sum_p)) return fail(CDD_EINVAL, "instance not usable for UCDDCP (no m/gamma, data too large for the packed records, or d < sum p)");
+    DeviceGuard g(I->device);
+    cudaError_t e = cdd::launch_schedule(*I, ucd, perms, ld, batch, C, X, start, penalty, as_stream(stream));
+    return e == cudaSuccess ? CDD_OK : cuda_fail(e, "cdd_schedule_batch");
+}
+
 int cdd_eval_batch_host(cdd_instance* I, cdd_problem problem, const int16_t* perms_host, int64_t ld,
                         int64_t batch, int64_t* out_host, void* stream) {
     int rc = check_batch_args(I, perms_host, ld, batch, out_host);

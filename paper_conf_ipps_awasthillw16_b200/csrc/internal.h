@@ -52,6 +52,11 @@ struct Instance {
 cudaError_t launch_eval_batch(const Instance& I, bool ucd, const int16_t* perms, int64_t ld,
                               int64_t batch, int64_t* out, cudaStream_t s);
 
+// ---- launchers (schedule.cu) ----
+cudaError_t launch_schedule(const Instance& I, bool ucd, const int16_t* perms, int64_t ld,
+                            int64_t batch, int64_t* C, int32_t* X, int64_t* start, int64_t* pen,
+                            cudaStream_t s);
+
 // ---- launchers (sa.cu) ----
 struct SaLaunch {
     bool ucd;
