@@ -81,6 +81,7 @@ def _load():
             "or_t0": (dbl, [vp, i32, u64, i64]),
             "or_sa_chain": (i64, [vp, vp, dbl, u64, vp, vp, vp, vp]),
             "or_sa_run": (None, [vp, vp, dbl, vp, vp, vp, vp]),
+            "or_sa_sync": (None, [vp, vp, dbl, i64, vp, vp, vp, vp, vp, vp]),
             "or_dpso_f1": (None, [i32, vp, u32, u32, vp]),
             "or_dpso_f2": (None, [i32, vp, vp, u32, vp]),
             "or_dpso_f3": (None, [i32, vp, vp, u32, u32, vp]),
@@ -230,6 +231,19 @@ def sa_chain(prob: Problem, p: SAParams, T0: float, g: int, trace: bool = False)
         res["E_new"] = tr >> 1
         res["accepted"] = (tr & 1).astype(bool)
     return res
+
+
+def sa_sync(prob: Problem, p: SAParams, T0: float, levels: int):
+    """Synchronous SA: p.steps = Markov-chain length M per temperature level."""
+    n = prob.n
+    bE, bg, bl = C.c_int64(), C.c_uint64(), C.c_int64()
+    J = np.zeros(n, dtype=np.int16)
+    lE = np.zeros(levels, dtype=np.int64)
+    lg = np.zeros(levels, dtype=np.uint64)
+    _load().or_sa_sync(prob.ref, C.byref(p), T0, levels, C.byref(bE), C.byref(bg), C.byref(bl),
+                       _ptr(J), _ptr(lE), _ptr(lg))
+    return {"E_best": bE.value, "g": bg.value, "level": bl.value, "best": J, "level_min_E": lE,
+            "level_min_g": lg}
 
 
 def sa_run(prob: Problem, p: SAParams, T0: float, chain_best: bool = False):

@@ -201,6 +201,49 @@ def test_sa_n10_reaches_the_nfact_optimum():
     assert r["E_best"] == z_opt
 
 
+# ---------------------------------------------------------------------- synchronous SA (F2)
+def test_sa_sync_single_chain_unit_length_is_the_async_chain():
+    # chains = 1, M = 1: level j is one move at T0*mu^j from the previous final state with the
+    # counters of step j -- exactly Alg. 1 (cooling every step)
+    inst, pr, p = _sa(n=40, steps=1, seed=5)
+    T0 = oracle.t0(pr, oracle.CDD, 5, 400)
+    L = 700
+    s = oracle.sa_sync(pr, p, T0, L)
+    pa = oracle.sa_params(chains=1, steps=L, seed=5)
+    a = oracle.sa_chain(pr, pa, T0, 0, trace=True)
+    assert s["E_best"] == a["E_best"] and s["g"] == 0
+    assert oracle.cdd_eval(pr, s["best"]) == s["E_best"]
+    # the level minimum is the chain's state after each step
+    E, states = oracle.cdd_eval(pr, oracle.perm_fy(inst.n, 5, oracle.TAG_SA_INIT, 0)), []
+    for En, acc in zip(a["E_new"], a["accepted"]):
+        E = int(En) if acc else E
+        states.append(E)
+    assert np.array_equal(s["level_min_E"], np.array(states))
+
+
+def test_sa_sync_one_level_is_async_at_constant_temperature():
+    inst, pr, p = _sa(n=30, steps=250, seed=9, chains=10, chain_offset=7)
+    r = oracle.sa_sync(pr, p, 60.0, 1)
+    pa = oracle.sa_params(chains=10, steps=250, seed=9, chain_offset=7, mu=1.0)
+    a = oracle.sa_run(pr, pa, 60.0)
+    assert (r["E_best"], r["g"]) == (a["E_best"], a["g"]) and np.array_equal(r["best"], a["best"])
+    finals = [oracle.sa_chain(pr, pa, 60.0, 7 + c)["E_final"] for c in range(10)]
+    assert r["level_min_E"][0] == min(finals) and r["level_min_g"][0] == 7 + int(np.argmin(finals))
+
+
+def test_sa_sync_greedy_levels_never_worsen_and_n10_optimum():
+    inst, pr, p = _sa(n=25, steps=40, seed=3, chains=8)
+    r = oracle.sa_sync(pr, p, 0.0, 30)  # T = 0: only non-worsening moves
+    assert np.all(np.diff(r["level_min_E"]) <= 0)
+    assert r["E_best"] == r["level_min_E"].min() == oracle.cdd_eval(pr, r["best"])
+    inst = gen.cdd_instance(10, 1, 0.4)
+    pr = oracle.Problem.from_instance(inst)
+    z_opt = int(oracle.eval_batch_threaded(pr, gen.all_perms(10)).min())
+    p = oracle.sa_params(chains=32, steps=20, seed=0x5EED0002)
+    r = oracle.sa_sync(pr, p, oracle.t0(pr, oracle.CDD, 0x5EED0002), 60)
+    assert r["E_best"] == z_opt
+
+
 # ----------------------------------------------------------------------------------- DPSO
 def test_dpso_operators():
     rng = np.random.default_rng(3)
