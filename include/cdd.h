@@ -157,6 +157,48 @@ CDD_API int sa_t0(cdd_instance *inst, cdd_problem problem, uint64_t seed, int64_
           void *workspace, size_t workspace_bytes, void *stream);
 
 /* ------------------------------------------------------------------------------------------ */
+/* Synchronous SA (Fig. 8; reading R18)                                   */
+/* ------------------------------------------------------------------------------------------ */
+/* Every chain starts from its own random state; at temperature level j = 0..levels-1 every chain
+ * runs a Markov chain of markov_len (M) moves at the constant temperature T_j (T_0 from T0 /
+ * t0_samples / T0_in as in sa_params, T_{j+1} = T_j * mu); the final state of minimal penalty over
+ * all chains (ties: lowest global id) is the initial state of every chain at level j+1.  Move m of
+ * level j uses the Philox counters of step j*M + m.  The instance's best buffers receive the
+ * best-ever state (within a level min (penalty, chain id); a later level only if strictly better).
+ * Runs on the group layout (lanes 0 = automatic, 4, 8, 16; needs alpha, beta <= 255). */
+typedef struct {
+    cdd_problem problem;
+    int64_t chains;        /* chains on this device                                            */
+    int64_t markov_len;    /* M: moves per chain per temperature level (>= 1)                  */
+    int64_t levels;        /* temperature levels (>= 1); levels * M < 2^32                      */
+    double mu;             /* cooling factor between levels                                      */
+    double T0;             /* > 0: initial temperature; <= 0: from t0_samples             */
+    int64_t t0_samples;
+    int32_t pert;          /* 1 <= pert <= 4                                                     */
+    cdd_move move;
+    uint64_t seed;
+    uint64_t chain_offset; /* global id of local chain 0 (multi-GPU: rank * chains)              */
+    int32_t lanes;         /* threads per chain: 0 automatic, 4, 8 or 16                         */
+    double *T0_out;        /* optional device double [1]: T_0                                    */
+    const double *T0_in;   /* optional device double [1]: T_0 read on the device                */
+    int64_t *level_min;    /* optional device int64 [levels]: penalty of s^min_j (device-local)  */
+} sa_sync_params;
+CDD_API size_t sa_sync_workspace_size(const cdd_instance *inst, const sa_sync_params *params);
+/* ASYNC.  All levels on this device (the swarm of chains is this device's). */
+CDD_API int sa_sync_run(cdd_instance *inst, const sa_sync_params *params, void *workspace,
+                        size_t workspace_bytes, void *stream);
+/* Stepping interface for chains spread over several GPUs.  ASYNC.  sa_sync_level(j) runs level j
+ * (call j = 0, 1, ..., levels-1 in order with the same workspace); afterwards sa_sync_ptrs gives
+ * the level's packed key (final penalty << 32 | global id, int64) and the int16 [n] state s^min_j
+ * that level j+1 starts from -- MIN-all-reduce the key and broadcast the state from the owning
+ * rank between levels; the best-ever buffers stay device-local (reduce them with the async-SA
+ * helpers at the end). */
+CDD_API int sa_sync_level(cdd_instance *inst, const sa_sync_params *params, void *workspace,
+                          size_t workspace_bytes, int64_t j, void *stream);
+CDD_API int sa_sync_ptrs(const cdd_instance *inst, const sa_sync_params *params, void *workspace,
+                         int64_t **key_dev, int16_t **perm_dev);
+
+/* ------------------------------------------------------------------------------------------ */
 /* Discrete PSO (Alg. 2, eq. (3))                                                   */
 /* ------------------------------------------------------------------------------------------ */
 /* Operators (reading R15): F1 swaps two Floyd-sampled positions; F2 keeps the first

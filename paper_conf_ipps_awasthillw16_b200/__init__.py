@@ -46,6 +46,14 @@ class SaParams(C.Structure):
                 ("lanes", C.c_int32)]
 
 
+class SaSyncParams(C.Structure):
+    _fields_ = [("problem", C.c_int), ("chains", C.c_int64), ("markov_len", C.c_int64),
+                ("levels", C.c_int64), ("mu", C.c_double), ("T0", C.c_double),
+                ("t0_samples", C.c_int64), ("pert", C.c_int32), ("move", C.c_int),
+                ("seed", C.c_uint64), ("chain_offset", C.c_uint64), ("lanes", C.c_int32),
+                ("T0_out", C.c_void_p), ("T0_in", C.c_void_p), ("level_min", C.c_void_p)]
+
+
 class DpsoParams(C.Structure):
     _fields_ = [("problem", C.c_int), ("particles", C.c_int64), ("iters", C.c_int64),
                 ("w", C.c_double), ("c1", C.c_double), ("c2", C.c_double), ("seed", C.c_uint64),
@@ -66,6 +74,10 @@ _SIGS = {
     "sa_run": (C.c_int, [_vp, C.POINTER(SaParams), _vp, _sz, _vp]),
     "sa_t0": (C.c_int, [_vp, C.c_int, _u64, _i64, _vp, _vp, _sz, _vp]),
     "sa_layout": (C.c_int, [_vp, C.POINTER(SaParams), _vp, _vp]),
+    "sa_sync_workspace_size": (_sz, [_vp, C.POINTER(SaSyncParams)]),
+    "sa_sync_run": (C.c_int, [_vp, C.POINTER(SaSyncParams), _vp, _sz, _vp]),
+    "sa_sync_level": (C.c_int, [_vp, C.POINTER(SaSyncParams), _vp, _sz, _i64, _vp]),
+    "sa_sync_ptrs": (C.c_int, [_vp, C.POINTER(SaSyncParams), _vp, _vp, _vp]),
     "dpso_workspace_size": (_sz, [_vp, C.POINTER(DpsoParams)]),
     "dpso_run": (C.c_int, [_vp, C.POINTER(DpsoParams), _vp, _sz, _vp]),
     "dpso_begin": (C.c_int, [_vp, C.POINTER(DpsoParams), _vp, _sz, _vp]),
@@ -304,6 +316,51 @@ def sa_t0(inst: Instance, problem="cdd", seed=0, samples=5000, stream=None):
     return T0
 
 
+class SaSync:
+    """Synchronous SA on one GPU: `run()` does every level; `level(j)` and
+    `exchange_tensors()` let a caller share s^min across GPUs between levels."""
+
+    def __init__(self, inst: Instance, chains: int, markov_len: int, levels: int, problem="cdd",
+                 mu=0.88, T0=0.0, t0_samples=5000, pert=4, move="pert_fy", seed=0,
+                 chain_offset=0, lanes=0, level_min=True, T0_dev=None):
+        import torch
+
+        self.inst = inst
+        dev = torch.device("cuda", inst.device)
+        self.T0 = torch.empty(1, dtype=torch.float64, device=dev)
+        self.level_min = torch.empty(levels, dtype=torch.int64, device=dev) if level_min else None
+        self.p = SaSyncParams(PROBLEMS[problem], int(chains), int(markov_len), int(levels), float(mu),
+                              float(T0), int(t0_samples), int(pert), MOVES[move],
+                              int(seed) & (2**64 - 1), int(chain_offset), int(lanes),
+                              self.T0.data_ptr(), _dptr(T0_dev), _dptr(self.level_min))
+        need = int(_lib.sa_sync_workspace_size(inst.handle, C.byref(self.p)))
+        if need == 0:
+            _check(_lib.sa_sync_run(inst.handle, C.byref(self.p), None, 0, None))  # raises
+        self.ws = torch.empty(need, dtype=torch.uint8, device=dev)
+
+    def run(self, stream=None):
+        _check(_lib.sa_sync_run(self.inst.handle, C.byref(self.p), self.ws.data_ptr(),
+                                self.ws.numel(), _stream(stream)))
+        return self
+
+    def level(self, j: int, stream=None):
+        _check(_lib.sa_sync_level(self.inst.handle, C.byref(self.p), self.ws.data_ptr(),
+                                  self.ws.numel(), int(j), _stream(stream)))
+
+    def exchange_tensors(self):
+        """(key int64 [1], s^min int16 [n]) device views for the between-level exchange."""
+        k, q = _vp(), _vp()
+        _check(_lib.sa_sync_ptrs(self.inst.handle, C.byref(self.p), self.ws.data_ptr(),
+                                 C.byref(k), C.byref(q)))
+        return (_device_view(k.value, (1,), "<i8", self.inst.device),
+                _device_view(q.value, (self.inst.n,), "<i2", self.inst.device))
+
+
+def sa_sync_run(inst: Instance, chains: int, markov_len: int, levels: int, **kw) -> SaSync:
+    """Synchronous SA on one GPU; the best-ever state goes to the instance's best buffers."""
+    return SaSync(inst, chains, markov_len, levels, **kw).run()
+
+
 class Dpso:
     """A DPSO swarm on one GPU (Alg. 2, eq. (3)).  `run()` does the whole single-GPU run; the
     stepping methods let a caller exchange the swarm best across GPUs between iterations."""
@@ -371,6 +428,12 @@ class _CudaArray:
     def __init__(self, ptr, shape, typestr):
         self.__cuda_array_interface__ = {"shape": shape, "typestr": typestr, "data": (ptr, False),
                                          "version": 3, "strides": None}
+
+
+def _device_view(ptr, shape, typestr, device):
+    import torch
+
+    return torch.as_tensor(_CudaArray(ptr, shape, typestr), device=torch.device("cuda", device))
 
 
 def best_device_tensors(inst: Instance):

@@ -369,6 +369,76 @@ size_t sa_workspace_size(const cdd_instance* I, const sa_params* p) {
     return cdd::sa_workspace_bytes(*I, L);
 }
 
+static int sync_validate(const cdd_instance* I, const sa_sync_params* q, cdd::SaLaunch* L) {
+    if (!I || !q) return fail(CDD_EINVAL, "instance/params is NULL");
+    if (q->markov_len < 1 || q->levels < 1) return fail(CDD_EINVAL, "markov_len and levels must be >= 1");
+    if ((double)q->markov_len * (double)q->levels >= 4294967296.0)
+        return fail(CDD_EINVAL, "levels * markov_len must be < 2^32");
+    if (q->lanes != 0 && q->lanes != 4 && q->lanes != 8 && q->lanes != 16)
+        return fail(CDD_EINVAL, "synchronous SA runs on lanes 0, 4, 8 or 16");
+    if (!I->ab16_ok) return fail(CDD_EINVAL, "synchronous SA needs alpha, beta <= 255 (16-bit records)");
+    sa_params p{};
+    p.problem = q->problem;
+    p.chains = q->chains;
+    p.steps = q->markov_len;
+    p.mu = q->mu;
+    p.T0 = q->T0;
+    p.t0_samples = q->t0_samples;
+    p.pert = q->pert;
+    p.move = q->move;
+    p.seed = q->seed;
+    p.chain_offset = q->chain_offset;
+    p.T0_out = q->T0_out;
+    p.T0_in = q->T0_in;
+    p.lanes = q->lanes;
+    return sa_validate(I, &p, L);
+}
+
+size_t sa_sync_workspace_size(const cdd_instance* I, const sa_sync_params* q) {
+    cdd::SaLaunch L{};
+    if (sync_validate(I, q, &L) != CDD_OK) return 0;
+    DeviceGuard g(I->device);
+    return cdd::sa_sync_workspace_bytes(*I, L);
+}
+
+int sa_sync_level(cdd_instance* I, const sa_sync_params* q, void* ws, size_t ws_bytes, int64_t j,
+                  void* stream) {
+    cdd::SaLaunch L{};
+    const int rc = sync_validate(I, q, &L);
+    if (rc != CDD_OK) return rc;
+    if (j < 0 || j >= q->levels) return fail(CDD_EINVAL, "level j out of range");
+    DeviceGuard g(I->device);
+    const size_t need = cdd::sa_sync_workspace_bytes(*I, L);
+    if (!ws || ws_bytes < need)
+        return fail(CDD_ENOMEM, "workspace too small: need " + std::to_string(need) + " bytes");
+    cudaError_t e = cdd::launch_sa_sync_level(*I, L, j, q->level_min, ws, as_stream(stream));
+    if (e != cudaSuccess) return cuda_fail(e, "sa_sync_level");
+    I->has_best = true;
+    return CDD_OK;
+}
+
+int sa_sync_run(cdd_instance* I, const sa_sync_params* q, void* ws, size_t ws_bytes, void* stream) {
+    for (int64_t j = 0; q && j < q->levels; ++j) {
+        const int rc = sa_sync_level(I, q, ws, ws_bytes, j, stream);
+        if (rc != CDD_OK) return rc;
+    }
+    return q ? CDD_OK : fail(CDD_EINVAL, "params is NULL");
+}
+
+int sa_sync_ptrs(const cdd_instance* I, const sa_sync_params* q, void* ws, int64_t** key_dev,
+                 int16_t** perm_dev) {
+    cdd::SaLaunch L{};
+    const int rc = sync_validate(I, q, &L);
+    if (rc != CDD_OK) return rc;
+    if (!ws) return fail(CDD_EINVAL, "workspace is NULL");
+    unsigned long long* k = nullptr;
+    int16_t* pp = nullptr;
+    cdd::sa_sync_ptrs(*I, L, ws, &k, &pp);
+    if (key_dev) *key_dev = reinterpret_cast<int64_t*>(k);
+    if (perm_dev) *perm_dev = pp;
+    return CDD_OK;
+}
+
 int sa_layout(const cdd_instance* I, const sa_params* p, int32_t* lanes, int32_t* positions_per_lane) {
     cdd::SaLaunch L{};
     const int rc = sa_validate(I, p, &L);

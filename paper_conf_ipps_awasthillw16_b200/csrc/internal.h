@@ -76,6 +76,12 @@ cudaError_t launch_t0(const Instance& I, bool ucd, uint64_t seed, int64_t sample
                       void* ws, cudaStream_t s);
 cudaError_t launch_sa(Instance& I, const SaLaunch& p, void* ws, cudaStream_t s);
 void sa_layout(const Instance& I, const SaLaunch& p, int32_t* lanes, int32_t* per_lane);
+// synchronous SA (p.steps = Markov-chain length M); 0 bytes if the instance has no 16-bit records
+size_t sa_sync_workspace_bytes(const Instance& I, const SaLaunch& p);
+cudaError_t launch_sa_sync_level(Instance& I, const SaLaunch& p, int64_t j, int64_t* level_min,
+                                 void* ws, cudaStream_t s);
+void sa_sync_ptrs(const Instance& I, const SaLaunch& p, void* ws, unsigned long long** key,
+                  int16_t** perm);
 
 // ---- launchers (dpso.cu) ----
 struct DpsoLaunch {

@@ -56,3 +56,21 @@ def dpso_run_distributed(inst, particles_per_rank: int, iters: int, problem="cdd
     reduce_best(key, perm, particles_per_rank, group)
     sw.end()
     return sw
+
+
+def sa_sync_run_distributed(inst, chains_per_rank: int, markov_len: int, levels: int, group=None,
+                            **kw):
+    """Synchronous SA over all ranks (global chain ids rank*C .. rank*C+C-1): after
+    every temperature level the minimal final state is global -- its packed key is MIN-all-reduced
+    and the state broadcast from its owner before the next level; the best-ever state is reduced
+    once at the end (global_best)."""
+    from . import SaSync
+
+    rank = dist.get_rank(group)
+    ss = SaSync(inst, chains_per_rank, markov_len, levels, chain_offset=rank * chains_per_rank, **kw)
+    for j in range(levels):
+        ss.level(j)
+        key, perm = ss.exchange_tensors()
+        reduce_best(key, perm, chains_per_rank, group)
+    global_best(inst, chains_per_rank, group)
+    return ss
