@@ -395,6 +395,18 @@ def bench_configs(lib, dev, stream):
                       "dpso_best": dpso_best, "sa_steps_equal_time": sa_steps, "sa_best": sa_best,
                       "workload": "CDD n=500 h=0.6, DPSO 8192 particles x 200 iterations (w=c1=c2=0.5) vs "
                                   "8192 SA chains for the same wall time, 1 GPU"}
+    # synchronous SA on the config-5 instance h=0.4: 65536 chains, M=50 x 100 levels
+    # (5000 moves per chain, like SA_5000) vs asynchronous SA with the same moves
+    i5 = lib.Instance.from_gen(gen.cdd_instance(N_JOBS, INSTANCE_SEED, 0.4), device=dev.index)
+    ss = lib.SaSync(i5, 65536, 50, 100, seed=RUN_SEED, t0_samples=T0_SAMPLES, level_min=False)
+    dt = _timed(stream, lambda: ss.run(), reps=1)
+    sync_best, _, _ = lib.best_get(i5)
+    lib.sa_run(i5, 65536, 5000, seed=RUN_SEED, t0_samples=T0_SAMPLES)
+    async_best, _, _ = lib.best_get(i5)
+    out["sync_sa"] = {"evals_per_s": 65536 * 5000 / dt, "ms": 1000 * dt, "best": sync_best,
+                      "async_best_same_moves": async_best,
+                      "workload": "synchronous SA, CDD n=1000 h=0.4, 65536 chains, M=50 moves x 100 "
+                                  "temperature levels (mu per level)"}
     return out
 
 
