@@ -415,6 +415,12 @@ cudaError_t dispatch(const Instance& I, const int16_t* perms, int64_t ld, int64_
 cudaError_t launch_eval_batch(const Instance& I, bool ucd, const int16_t* perms, int64_t ld,
                               int64_t batch, int64_t* out, cudaStream_t s) {
     if (batch <= 0) return cudaSuccess;
+#ifndef CDD_EVAL_V1
+    if (!ucd) {
+        const cudaError_t e = launch_eval2_cdd(I, perms, ld, batch, out, s);
+        if (e != cudaErrorNotSupported) return e;
+    }
+#endif
     return ucd ? dispatch<true>(I, perms, ld, batch, out, s)
                : dispatch<false>(I, perms, ld, batch, out, s);
 }

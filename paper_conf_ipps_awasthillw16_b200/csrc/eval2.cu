@@ -1,0 +1,311 @@
+// eval2.cu -- batched CDD evaluation, several sequences per warp (cdd_eval_batch, S§8 A2-A7).
+//
+// G lanes evaluate one sequence (32/G sequences per warp), lane l owns the E contiguous positions
+// [l*E, l*E+E).  Per warp, the job ids of the next group of sequences are copied from HBM to a
+// double-buffered shared-memory stage with cp.async (16-byte chunks, fully coalesced, no register
+// staging; chunk c of lane segment S lands in slot c ^ f(S) so that the lane-contiguous LDS.128
+// reads of a segment are bank-conflict free) while the current group is evaluated.  (A TMA bulk
+// copy per lane segment was measured slower: the copy takes uniform operands, so 32 per-lane
+// copies serialise into an ELECT/R2UR loop.)  The records are gathered from a
+// bank-partitioned table (8 copies, aligned to its size so a gather address is SHF + LOP3) into
+// registers as 16-bit alpha|beta<<8 pairs and p bytes, and the evaluation is the group kernel's
+// (sa_group.cuh): two scans, ballots, a boundary-row spread (re-gathered through the staged ids)
+// and the PRMT/IMAD/IDP.2A/IDP.4A pass -- 2 instructions per position.
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+#include "device_common.cuh"
+#include "internal.h"
+
+namespace cdd {
+namespace {
+
+constexpr int kE2Warps = 16;             // one 512-thread CTA per SM
+constexpr int kE2Threads = kE2Warps * 32;
+constexpr int kE2Copies = 8;             // table copies: lane L reads copy L % 8
+
+__device__ __forceinline__ uint32_t lds32(uint32_t addr) {
+    uint32_t v;
+    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(addr));
+    return v;
+}
+
+__device__ __forceinline__ uint4 lds128(uint32_t addr) {
+    uint4 v;
+    asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(addr));
+    return v;
+}
+
+__device__ __forceinline__ void cp_async16(uint32_t dst, const void* src) {
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(dst), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait1() { asm volatile("cp.async.wait_group 1;" ::: "memory"); }
+
+template <int G>
+__device__ __forceinline__ uint32_t gsum2(uint32_t v) {
+#pragma unroll
+    for (int off = G / 2; off > 0; off >>= 1) v += __shfl_xor_sync(kFull, v, off, G);
+    return v;
+}
+
+template <int G, int E>
+struct E2 {
+    static constexpr int CPW = 32 / G;        // sequences per warp
+    static constexpr int CPS = E / 8;         // 16-byte chunks per lane segment
+    static constexpr int ROWB = G * E * 2;    // staged bytes per sequence
+    static constexpr int STAGE = CPW * ROWB;
+    static constexpr int SPR = E / G;         // boundary-row positions per lane
+    static constexpr int T = (G * CPS + 31) / 32;  // chunks of one sequence per lane (at most)
+    // swizzle of lane segment S (numbered over the warp's sequences)
+    static __device__ __forceinline__ uint32_t sw(int S) { return (uint32_t)((S * CPS / 8) % CPS); }
+};
+
+// One group of 32/G sequences per warp and stage.
+template <int G, int E>
+__global__ void __launch_bounds__(kE2Threads, 1) eval2_cdd_kernel(
+    const uint16_t* __restrict__ tab_ab16, const uint8_t* __restrict__ tab_p, int n, int npow2,
+    int32_t d, const int16_t* __restrict__ perms, int64_t ld, int64_t batch,
+    int64_t* __restrict__ out, int* __restrict__ err) {
+    using X = E2<G, E>;
+    constexpr int CPW = X::CPW, CPS = X::CPS, SPR = X::SPR;
+    extern __shared__ __align__(16) uint8_t smem[];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const int grp = lane / G, l = lane % G, gbase = grp * G;
+    // stages (2 per warp), then the record table aligned to its own size
+    const uint32_t sbase = (uint32_t)__cvta_generic_to_shared(smem);
+    const uint32_t stage0 = sbase + (uint32_t)(warp * 2 * X::STAGE);
+    const uint32_t tbytes = (uint32_t)npow2 * 4u * kE2Copies;
+    const uint32_t traw = sbase + (uint32_t)(kE2Warps * 2 * X::STAGE);
+    const uint32_t tab = (traw + tbytes - 1u) & ~(tbytes - 1u);
+    uint32_t* s_tab = reinterpret_cast<uint32_t*>(smem + (tab - sbase));
+    for (int i = threadIdx.x; i < npow2 * kE2Copies; i += blockDim.x) {
+        const int id = i / kE2Copies;
+        s_tab[i] = id < n ? (uint32_t)__ldg(tab_ab16 + id) | ((uint32_t)__ldg(tab_p + id) << 16) : 0u;
+    }
+    __syncthreads();
+    constexpr int SH = 5;  // log2(4 bytes * 8 copies)
+    const uint32_t amask = tbytes - 4u * kE2Copies;
+    const uint32_t tabc = tab | (uint32_t)((lane % kE2Copies) * 4);
+
+    const int cpr = (n + 7) / 8;  // 16-byte chunks of real ids per sequence (ld % 8 == 0)
+    const int64_t ngroups = (batch + CPW - 1) / CPW;
+    const int64_t gstep = (int64_t)gridDim.x * kE2Warps;
+    // this lane copies chunks cg = lane + 32 t of every sequence of a group (its stage slot
+    // depends on the group only through nothing: the offsets are loop invariants)
+    auto issue = [&](int64_t rg, int st) {
+        const uint32_t sdst = stage0 + (uint32_t)(st * X::STAGE);
+#pragma unroll
+        for (int r = 0; r < CPW; ++r) {
+            const int64_t row = rg * CPW + r;
+            if (rg < ngroups && row < batch) {  // warp-uniform
+                const char* src = reinterpret_cast<const char*>(perms + row * ld) + lane * 16;
+#pragma unroll
+                for (int t = 0; t < X::T; ++t) {
+                    const int cg = lane + 32 * t, seg = cg / CPS, c = cg % CPS;
+                    const uint32_t slot = (uint32_t)(seg * CPS) + ((uint32_t)c ^ X::sw(r * G + seg));
+                    if (cg < cpr) cp_async16(sdst + (uint32_t)(r * X::ROWB) + 16u * slot, src + 512 * t);
+                }
+            }
+        }
+        cp_async_commit();
+    };
+
+    const int64_t rg0 = (int64_t)blockIdx.x * kE2Warps + warp;
+    issue(rg0, 0);
+    issue(rg0 + gstep, 1);
+    uint32_t vmax = 0;
+    bool bad = false;
+    const uint32_t s2 = (uint32_t)n * 0x10001u;  // two sentinel ids (zero records)
+    const uint32_t sw_own = X::sw(grp * G + l);
+    int it = 0;
+    for (int64_t rg = rg0; rg < ngroups; rg += gstep, ++it) {
+        const int st = it & 1;
+        cp_async_wait1();
+        __syncwarp();
+        const uint32_t srow = stage0 + (uint32_t)(st * X::STAGE) + (uint32_t)(grp * X::ROWB);
+        const int64_t row = rg * CPW + grp;
+        const bool rv = row < batch;
+        const int kmax = rv ? min(E, max(0, n - l * E)) : 0;  // valid positions in own segment
+        // ---- gather: 16-bit alpha|beta<<8 pairs and p bytes, lane totals
+        uint32_t abp[E / 2], pw[E / 4];
+        uint32_t tA = 0, tB = 0, tP = 0;
+        const uint32_t seg_addr = srow + (uint32_t)(l * CPS * 16);
+#pragma unroll
+        for (int c = 0; c < CPS; ++c) {
+            uint4 q = lds128(seg_addr + (((uint32_t)c ^ sw_own) << 4));
+            if (8 * c + 8 <= kmax) {
+                vmax = __vmaxu2(vmax, __vmaxu2(__vmaxu2(q.x, q.y), __vmaxu2(q.z, q.w)));
+            } else if (8 * c >= kmax) {  // wholly past n (or an idle row): zero records
+                q = make_uint4(s2, s2, s2, s2);
+            } else {  // the chunk straddling n (n % 8 != 0): check real ids, sentinel the rest
+                uint32_t ws[4] = {q.x, q.y, q.z, q.w};
+#pragma unroll
+                for (int j = 0; j < 4; ++j) {
+                    uint32_t lo = ws[j] & 0xffffu, hi = ws[j] >> 16;
+                    if (8 * c + 2 * j < kmax) bad |= lo >= (uint32_t)n; else lo = s2 & 0xffffu;
+                    if (8 * c + 2 * j + 1 < kmax) bad |= hi >= (uint32_t)n; else hi = s2 & 0xffffu;
+                    ws[j] = lo | (hi << 16);
+                }
+                q = make_uint4(ws[0], ws[1], ws[2], ws[3]);
+            }
+            const uint32_t wv[4] = {q.x, q.y, q.z, q.w};
+            uint32_t r[8];
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+                r[2 * j] = lds32(((wv[j] << SH) & amask) | tabc);
+                r[2 * j + 1] = lds32(((wv[j] >> (16 - SH)) & amask) | tabc);
+            }
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+                const uint32_t a = __byte_perm(r[2 * j], r[2 * j + 1], 0x5410u);
+                abp[4 * c + j] = a;
+                tA = __dp4a(a, 0x00010001u, tA);
+                tB = __dp4a(a, 0x01000100u, tB);
+            }
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+                const uint32_t p01 = __byte_perm(r[4 * h], r[4 * h + 1], 0x0062u);
+                const uint32_t p23 = __byte_perm(r[4 * h + 2], r[4 * h + 3], 0x0062u);
+                const uint32_t p4 = __byte_perm(p01, p23, 0x5410u);
+                pw[2 * c + h] = p4;
+                tP = __dp4a(p4, 0x01010101u, tP);
+            }
+        }
+        // ---- scans, boundary lanes (as gchain_eval_cdd)
+        const uint32_t tAB = tA | (tB << 16);
+        const uint32_t iP = group_incl_scan<G>(tP, 0);
+        const uint32_t iAB = group_incl_scan<G>(tAB, 0);
+        const int32_t Pb = (int32_t)(iP - tP);
+        const uint32_t ABb = iAB - tAB;
+        const int32_t Ab = (int32_t)(ABb & 0xffffu), Bb = (int32_t)(ABb >> 16);
+        const int32_t Btot = (int32_t)(__shfl_sync(kFull, iAB, G - 1, G) >> 16);
+        const bool lane_valid = l * E < n;
+        const int Lk = hibit(group_ballot<G>(lane_valid && (Ab + Bb <= Btot), gbase));
+        const int Lt = hibit(group_ballot<G>(lane_valid && (Pb <= d), gbase));
+        const int Ls = max(0, min(Lk, Lt));
+        const int32_t PbS = __shfl_sync(kFull, Pb, Ls, G);
+        const uint32_t ABbS = __shfl_sync(kFull, ABb, Ls, G);
+        const int32_t thr = Btot - (int32_t)(ABbS & 0xffffu) - (int32_t)(ABbS >> 16);
+        const uint32_t key = ((uint32_t)min(thr, 0xffff) << 16) | 0xffffu;
+        // boundary row Ls: SPR consecutive positions per lane, re-gathered through the staged ids
+        const int e0 = l * SPR;
+        uint32_t idw[(SPR + 1) / 2];
+        {
+            const uint32_t bseg = srow + (uint32_t)(Ls * CPS * 16);
+            const uint32_t bsw = X::sw(grp * G + Ls);
+            if constexpr (SPR >= 8) {
+#pragma unroll
+                for (int v = 0; v < SPR / 8; ++v) {
+                    const uint4 q = lds128(bseg + ((((uint32_t)(e0 / 8 + v)) ^ bsw) << 4));
+                    idw[4 * v] = q.x; idw[4 * v + 1] = q.y; idw[4 * v + 2] = q.z; idw[4 * v + 3] = q.w;
+                }
+            } else {
+                const uint32_t a = bseg + ((((uint32_t)(e0 / 8)) ^ bsw) << 4) + (uint32_t)((e0 % 8) * 2);
+                if constexpr (SPR == 4) {
+                    uint32_t x0, x1;
+                    asm volatile("ld.shared.v2.u32 {%0,%1}, [%2];" : "=r"(x0), "=r"(x1) : "r"(a));
+                    idw[0] = x0; idw[1] = x1;
+                } else if constexpr (SPR == 2) {
+                    idw[0] = lds32(a);
+                } else {
+                    uint32_t x;
+                    asm volatile("ld.shared.u16 %0, [%1];" : "=r"(x) : "r"(a));
+                    idw[0] = x;
+                }
+            }
+        }
+        uint32_t v[SPR];
+        uint32_t lsum = 0;
+        const int kb = Ls * E + e0;  // sequence position of this lane's first boundary element
+#pragma unroll
+        for (int i = 0; i < SPR; ++i) {
+            const uint32_t id = (i & 1) ? (idw[i >> 1] >> 16) : (idw[i >> 1] & 0xffffu);
+            const uint32_t rec = (rv && kb + i < n) ? lds32(((id << SH) & amask) | tabc) : 0u;
+            // p | (alpha + beta) << 16
+            v[i] = __byte_perm(rec, 0u, 0x4442u) + (__dp4a(rec, 0x00000101u, 0u) << 16);
+            lsum += v[i];
+        }
+        const uint32_t ex = group_incl_scan<G>(lsum, 0) - lsum;
+        uint32_t run = ex, cinc = 0;
+        const bool sat0 = ex <= key;
+#pragma unroll
+        for (int i = 0; i < SPR; ++i) {
+            const bool sat = run <= key;
+            run += v[i];
+            cinc = sat ? run : cinc;
+        }
+        const int own = max(0, hibit(group_ballot<G>(sat0, gbase)));
+        const int32_t Ck0 = PbS + (int32_t)(__shfl_sync(kFull, cinc, own, G) & 0xffffu);
+        const int32_t Dr = ((Ls == Lk) ? min(Ck0, d) : d) - PbS;
+        int32_t corr = 0;
+        run = ex;
+#pragma unroll
+        for (int i = 0; i < SPR; ++i) {
+            const int32_t ci = (int32_t)(run & 0xffffu), si = (int32_t)(run >> 16);
+            corr += (si - thr) * min((int32_t)(v[i] & 0xffu), max(0, Dr - ci));
+            run += v[i];
+        }
+        __syncwarp();  // every lane is done with the stage: refill it two groups ahead
+        issue(rg + 2 * gstep, st);
+        // ---- F(C_m'): early weights left of lane Ls, tardy weights from it on
+        const bool amode = l < Ls;
+        const uint32_t psel = amode ? 0x4044u : 0x4144u;
+        const uint32_t wsum = amode ? 0x00010001u : 0x01000100u;
+        uint32_t s = 0, acc = 0;
+#pragma unroll
+        for (int j = 0; j < E / 2; ++j) {
+            const uint32_t f2 = s * 0x10001u + __byte_perm(abp[j], 0u, psel);
+            acc = (j & 1) ? __dp2a_hi(f2, pw[j >> 1], acc) : __dp2a_lo(f2, pw[j >> 1], acc);
+            s = __dp4a(abp[j], wsum, s);
+        }
+        const int32_t base = amode ? Ab : (Btot - Bb);
+        const int32_t contrib = base * (int32_t)tP + (amode ? (int32_t)acc : -(int32_t)acc) + corr;
+        const int32_t Z = (int32_t)gsum2<G>((uint32_t)contrib);
+        if (rv && l == 0) out[row] = (int64_t)Z;
+    }
+    asm volatile("cp.async.wait_all;" ::: "memory");
+    if (bad || (vmax & 0xffffu) >= (uint32_t)n || (vmax >> 16) >= (uint32_t)n) atomicOr(err, 1);
+}
+
+template <int G, int E>
+cudaError_t launch2(const Instance& I, const int16_t* perms, int64_t ld, int64_t batch,
+                    int64_t* out, cudaStream_t s) {
+    using X = E2<G, E>;
+    int npow2 = 1;
+    while (npow2 <= I.n) npow2 <<= 1;
+    const size_t tbytes = (size_t)npow2 * 4 * kE2Copies;
+    const size_t smem = (size_t)kE2Warps * 2 * X::STAGE + 2 * tbytes;  // room to align the table
+    auto kern = eval2_cdd_kernel<G, E>;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    int sms = 148;
+    e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, I.device);
+    if (e != cudaSuccess) return e;
+    const int64_t groups = (batch + X::CPW - 1) / X::CPW;
+    int64_t blocks = (groups + kE2Warps - 1) / kE2Warps;
+    if (blocks > sms) blocks = sms;
+    if (blocks < 1) blocks = 1;
+    kern<<<(unsigned)blocks, kE2Threads, smem, s>>>(I.tab_ab16, I.tab_p, I.n, npow2, I.d_eff, perms,
+                                                    ld, batch, out, I.err);
+    return cudaGetLastError();
+}
+
+}  // namespace
+
+// Returns cudaErrorNotSupported when the layout does not apply (the caller falls back).
+cudaError_t launch_eval2_cdd(const Instance& I, const int16_t* perms, int64_t ld, int64_t batch,
+                             int64_t* out, cudaStream_t s) {
+    if (!I.ab16_ok || ld % 8 != 0 || (reinterpret_cast<uintptr_t>(perms) & 15) != 0 || I.n > 1023)
+        return cudaErrorNotSupported;  // n = 1024 would need a 2048-entry table (64 KB x 2)
+    const int n = I.n;
+    if (n <= 16) return cudaErrorNotSupported;  // one-warp-per-many-rows kernel of eval.cu is faster
+    if (n <= 64) return launch2<4, 16>(I, perms, ld, batch, out, s);
+    if (n <= 128) return launch2<4, 32>(I, perms, ld, batch, out, s);
+    if (n <= 256) return launch2<8, 32>(I, perms, ld, batch, out, s);
+    if (n <= 512) return launch2<8, 64>(I, perms, ld, batch, out, s);
+    return launch2<16, 64>(I, perms, ld, batch, out, s);
+}
+
+}  // namespace cdd

@@ -52,6 +52,11 @@ struct Instance {
 cudaError_t launch_eval_batch(const Instance& I, bool ucd, const int16_t* perms, int64_t ld,
                               int64_t batch, int64_t* out, cudaStream_t s);
 
+// ---- launchers (eval2.cu): CDD, several sequences per warp; cudaErrorNotSupported if the
+// layout does not apply (alpha or beta > 255, ld % 8 != 0, rows not 16-byte aligned)
+cudaError_t launch_eval2_cdd(const Instance& I, const int16_t* perms, int64_t ld, int64_t batch,
+                             int64_t* out, cudaStream_t s);
+
 // ---- launchers (schedule.cu) ----
 cudaError_t launch_schedule(const Instance& I, bool ucd, const int16_t* perms, int64_t ld,
                             int64_t batch, int64_t* C, int32_t* X, int64_t* start, int64_t* pen,
