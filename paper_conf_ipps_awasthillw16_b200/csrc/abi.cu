@@ -207,6 +207,7 @@ int cdd_instance_create(int32_t n, const int32_t* p, const int32_t* alpha, const
         chk(cudaMemset(I->err, 0, sizeof(int)));
         chk(cudaMemset(I->best_key, 0xff, sizeof(unsigned long long)));
         chk(cudaMemset(I->best_perm, 0, sizeof(int16_t) * n));
+        chk(cdd::probe_smem_base(&I->smem_base));
     }
     if (e != cudaSuccess) {
         free_instance(I);

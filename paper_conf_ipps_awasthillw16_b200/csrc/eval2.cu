@@ -23,7 +23,22 @@ namespace {
 
 constexpr int kE2Warps = 16;             // one 512-thread CTA per SM
 constexpr int kE2Threads = kE2Warps * 32;
-constexpr int kE2Copies = 8;             // table copies: lane L reads copy L % 8
+// Table copies KC: lane L reads copy L % KC; 16 copies (2-way-at-worst bank conflicts between
+// lanes L and L+16) when shared memory allows, else 8 (4 lanes per copy, ~2.9 wavefronts/gather).
+constexpr int kE2MaxSmem = 227 * 1024;
+
+// Shared-memory layout: the table (KC copies x npow2 words) must sit at an address aligned to its
+// size (a gather address is then SHF + LOP3); the per-warp stages fill the gap below it first
+// (the dynamic window starts above a reserved 1 KB), the rest go above it.
+struct E2Layout {
+    uint32_t tab_off, nb, total;  // offsets from the dynamic base; nb = warps placed below
+};
+__host__ __device__ inline E2Layout e2_layout(uint32_t sbase, uint32_t tbytes, uint32_t wbytes, int W) {
+    const uint32_t tab = (sbase + tbytes - 1u) / tbytes * tbytes;
+    uint32_t nb = (tab - sbase) / wbytes;
+    if (nb > (uint32_t)W) nb = (uint32_t)W;
+    return {tab - sbase, nb, tab + tbytes + ((uint32_t)W - nb) * wbytes - sbase};
+}
 
 __device__ __forceinline__ uint32_t lds32(uint32_t addr) {
     uint32_t v;
@@ -66,28 +81,29 @@ struct E2 {
 template <int G, int E>
 __global__ void __launch_bounds__(kE2Threads, 1) eval2_cdd_kernel(
     const uint16_t* __restrict__ tab_ab16, const uint8_t* __restrict__ tab_p, int n, int npow2,
-    int32_t d, const int16_t* __restrict__ perms, int64_t ld, int64_t batch,
+    int kc_log2, int32_t d, const int16_t* __restrict__ perms, int64_t ld, int64_t batch,
     int64_t* __restrict__ out, int* __restrict__ err) {
     using X = E2<G, E>;
     constexpr int CPW = X::CPW, CPS = X::CPS, SPR = X::SPR;
     extern __shared__ __align__(16) uint8_t smem[];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const int grp = lane / G, l = lane % G, gbase = grp * G;
-    // stages (2 per warp), then the record table aligned to its own size
+    const int KC = 1 << kc_log2;
     const uint32_t sbase = (uint32_t)__cvta_generic_to_shared(smem);
-    const uint32_t stage0 = sbase + (uint32_t)(warp * 2 * X::STAGE);
-    const uint32_t tbytes = (uint32_t)npow2 * 4u * kE2Copies;
-    const uint32_t traw = sbase + (uint32_t)(kE2Warps * 2 * X::STAGE);
-    const uint32_t tab = (traw + tbytes - 1u) & ~(tbytes - 1u);
-    uint32_t* s_tab = reinterpret_cast<uint32_t*>(smem + (tab - sbase));
-    for (int i = threadIdx.x; i < npow2 * kE2Copies; i += blockDim.x) {
-        const int id = i / kE2Copies;
+    const uint32_t tbytes = (uint32_t)npow2 * 4u * (uint32_t)KC;
+    const E2Layout Ly = e2_layout(sbase, tbytes, 2u * X::STAGE, kE2Warps);
+    const uint32_t tab = sbase + Ly.tab_off;
+    const uint32_t stage0 = sbase + ((uint32_t)warp < Ly.nb ? (uint32_t)warp * 2u * X::STAGE
+                                                              : Ly.tab_off + tbytes + ((uint32_t)warp - Ly.nb) * 2u * X::STAGE);
+    uint32_t* s_tab = reinterpret_cast<uint32_t*>(smem + Ly.tab_off);
+    for (int i = threadIdx.x; i < npow2 * KC; i += blockDim.x) {
+        const int id = i >> kc_log2;
         s_tab[i] = id < n ? (uint32_t)__ldg(tab_ab16 + id) | ((uint32_t)__ldg(tab_p + id) << 16) : 0u;
     }
     __syncthreads();
-    constexpr int SH = 5;  // log2(4 bytes * 8 copies)
-    const uint32_t amask = tbytes - 4u * kE2Copies;
-    const uint32_t tabc = tab | (uint32_t)((lane % kE2Copies) * 4);
+    const int SH = 2 + kc_log2;  // log2(4 bytes * KC copies)
+    const uint32_t amask = tbytes - 4u * (uint32_t)KC;
+    const uint32_t tabc = tab | (uint32_t)((lane & (KC - 1)) * 4);
 
     const int cpr = (n + 7) / 8;  // 16-byte chunks of real ids per sequence (ld % 8 == 0)
     const int64_t ngroups = (batch + CPW - 1) / CPW;
@@ -275,8 +291,14 @@ cudaError_t launch2(const Instance& I, const int16_t* perms, int64_t ld, int64_t
     using X = E2<G, E>;
     int npow2 = 1;
     while (npow2 <= I.n) npow2 <<= 1;
-    const size_t tbytes = (size_t)npow2 * 4 * kE2Copies;
-    const size_t smem = (size_t)kE2Warps * 2 * X::STAGE + 2 * tbytes;  // room to align the table
+    int kc_log2 = 4;
+    E2Layout Ly = e2_layout(I.smem_base, (uint32_t)npow2 * 4u << kc_log2, 2u * X::STAGE, kE2Warps);
+    if (Ly.total > (uint32_t)kE2MaxSmem) {
+        kc_log2 = 3;
+        Ly = e2_layout(I.smem_base, (uint32_t)npow2 * 4u << kc_log2, 2u * X::STAGE, kE2Warps);
+    }
+    if (Ly.total > (uint32_t)kE2MaxSmem) return cudaErrorNotSupported;
+    const size_t smem = Ly.total;
     auto kern = eval2_cdd_kernel<G, E>;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
@@ -287,18 +309,33 @@ cudaError_t launch2(const Instance& I, const int16_t* perms, int64_t ld, int64_t
     int64_t blocks = (groups + kE2Warps - 1) / kE2Warps;
     if (blocks > sms) blocks = sms;
     if (blocks < 1) blocks = 1;
-    kern<<<(unsigned)blocks, kE2Threads, smem, s>>>(I.tab_ab16, I.tab_p, I.n, npow2, I.d_eff, perms,
-                                                    ld, batch, out, I.err);
+    kern<<<(unsigned)blocks, kE2Threads, smem, s>>>(I.tab_ab16, I.tab_p, I.n, npow2, kc_log2, I.d_eff,
+                                                    perms, ld, batch, out, I.err);
     return cudaGetLastError();
+}
+
+__global__ void smem_base_probe(uint32_t* out) {
+    extern __shared__ __align__(16) uint8_t smem[];
+    *out = (uint32_t)__cvta_generic_to_shared(smem);
 }
 
 }  // namespace
 
+cudaError_t probe_smem_base(uint32_t* base) {
+    uint32_t* d = nullptr;
+    cudaError_t e = cudaMalloc(&d, sizeof(uint32_t));
+    if (e != cudaSuccess) return e;
+    smem_base_probe<<<1, 1, 16>>>(d);
+    e = cudaMemcpy(base, d, sizeof(uint32_t), cudaMemcpyDeviceToHost);
+    cudaFree(d);
+    return e;
+}
+
 // Returns cudaErrorNotSupported when the layout does not apply (the caller falls back).
 cudaError_t launch_eval2_cdd(const Instance& I, const int16_t* perms, int64_t ld, int64_t batch,
                              int64_t* out, cudaStream_t s) {
-    if (!I.ab16_ok || ld % 8 != 0 || (reinterpret_cast<uintptr_t>(perms) & 15) != 0 || I.n > 1023)
-        return cudaErrorNotSupported;  // n = 1024 would need a 2048-entry table (64 KB x 2)
+    if (!I.ab16_ok || ld % 8 != 0 || (reinterpret_cast<uintptr_t>(perms) & 15) != 0)
+        return cudaErrorNotSupported;
     const int n = I.n;
     if (n <= 16) return cudaErrorNotSupported;  // one-warp-per-many-rows kernel of eval.cu is faster
     if (n <= 64) return launch2<4, 16>(I, perms, ld, batch, out, s);

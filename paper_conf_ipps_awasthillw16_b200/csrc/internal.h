@@ -34,6 +34,7 @@ struct Instance {
     uint32_t* tab_ab = nullptr;
     uint16_t* tab_ab16 = nullptr;  // alpha | beta << 8 (only when both <= 255: ab16_ok)
     bool ab16_ok = false;
+    uint32_t smem_base = 1024;  // shared-window address of dynamic shared memory (probed at create)
     uint8_t* tab_p = nullptr;
     uint8_t* tab_m = nullptr;
     uint8_t* tab_x = nullptr;
@@ -56,6 +57,7 @@ cudaError_t launch_eval_batch(const Instance& I, bool ucd, const int16_t* perms,
 // layout does not apply (alpha or beta > 255, ld % 8 != 0, rows not 16-byte aligned)
 cudaError_t launch_eval2_cdd(const Instance& I, const int16_t* perms, int64_t ld, int64_t batch,
                              int64_t* out, cudaStream_t s);
+cudaError_t probe_smem_base(uint32_t* base);
 
 // ---- launchers (schedule.cu) ----
 cudaError_t launch_schedule(const Instance& I, bool ucd, const int16_t* perms, int64_t ld,

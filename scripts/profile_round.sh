@@ -7,6 +7,6 @@ ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpuru
     python bench.py --steps 1 --warmup 0 --no-cpu-baseline --no-e2e --no-eval --no-configs > /dev/null 2>&1
 ncu --set full --clock-control none --import-source on -k regex:sa_group -c 1 -o gpurun_out/prof_sa_full \
     python bench.py --steps 1 --warmup 0 --no-cpu-baseline --no-e2e --no-eval --no-configs > /dev/null 2>&1
-ncu --set full --clock-control none --import-source on -k regex:eval_batch -s 3 -c 1 -o gpurun_out/prof_eval_full \
-    python bench.py --steps 1 --warmup 0 --sa-steps 10 --chains 1024 --no-cpu-baseline --no-e2e > /dev/null 2>&1
+ncu --set full --clock-control none --import-source on -k regex:eval -s 1 -c 1 -o gpurun_out/prof_eval_full \
+    python scripts/eval_sweep.py --reps 2 1000 > /dev/null 2>&1
 ls -la gpurun_out
