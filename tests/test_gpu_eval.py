@@ -140,16 +140,24 @@ def test_large_n_row_strides(lib, n, pad):
             assert np.array_equal(_gpu_eval(lib, inst, perms, d=d), _oracle(inst, perms, d=d)), (n, ld, h)
 
 
-def test_invalid_ids_flagged(lib):
-    inst = gen.cdd_instance(50, 1, 0.4)
-    perms = gen.random_perms(10, 50, 1)
-    perms[3, 7] = 50
+@pytest.mark.parametrize("n", [10, 50, 201, 500, 1000, 1023])
+@pytest.mark.parametrize("problem", ["cdd", "ucddcp"])
+def test_invalid_ids_flagged(lib, n, problem):
+    inst = gen.ucddcp_instance(n, 1) if problem == "ucddcp" else gen.cdd_instance(n, 1, 0.4)
     ins = lib.Instance.from_gen(inst)
-    lib.cdd_eval_batch(ins, _dev(perms))
-    with pytest.raises(lib.CddError) as e:
-        lib.cdd_check(ins)
-    assert e.value.code == lib.CDD_EDATA
-    lib.cdd_check(ins)  # flag cleared
+    fn = lib.ucddcp_eval_batch if problem == "ucddcp" else lib.cdd_eval_batch
+    perms = gen.random_perms(70, n, 1)
+    fn(ins, _dev(perms))
+    lib.cdd_check(ins)  # valid rows: no flag
+    npow2 = 1 << n.bit_length()
+    for bad, pos in [(n, 7 % n), (npow2 - 1, n - 1), (32767, n // 2), (-1, 0)]:
+        q = perms.copy()
+        q[69 if bad == n else 3, pos] = bad
+        fn(ins, _dev(q))
+        with pytest.raises(lib.CddError) as e:
+            lib.cdd_check(ins)
+        assert e.value.code == lib.CDD_EDATA
+        lib.cdd_check(ins)  # flag cleared
 
 
 def test_host_e2e_path(lib):

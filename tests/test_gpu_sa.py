@@ -246,3 +246,28 @@ def test_sa_layout_query(lib):
         assert g in (4, 8, 16, 32) and g * e >= n and (lanes == 0 or g == lanes)
         if chains < 1024:
             assert g == 32
+
+
+def test_bench_config_sampled_parity(lib):
+    # the BASELINE headline configuration exactly as bench.py launches it (config 5, h = 0.4:
+    # n = 1000, 65536 chains x 5000 steps, T0 from 5000 samples, automatic layout); the oracle
+    # replays sampled chains one by one, the global best is re-evaluated
+    import torch
+
+    import bench
+
+    inst = gen.cdd_instance(bench.N_JOBS, bench.INSTANCE_SEED, 0.4)
+    ins = lib.Instance.from_gen(inst)
+    T0 = lib.sa_t0(ins, "cdd", seed=bench.RUN_SEED, samples=bench.T0_SAMPLES)
+    res = lib.sa_run(ins, bench.CHAINS, bench.SA_STEPS, seed=bench.RUN_SEED, T0_dev=T0,
+                     chain_best=True)
+    torch.cuda.synchronize()
+    pen, perm, gid = lib.best_get(ins)
+    cb = res["chain_best"].cpu().numpy()
+    pr = _prob(inst)
+    assert oracle.cdd_eval(pr, perm) == pen == cb.min() and gid == int(np.argmin(cb))
+    T0v = float(T0.item())
+    assert T0v == oracle.t0(pr, oracle.CDD, bench.RUN_SEED, bench.T0_SAMPLES)
+    p = oracle.sa_params(chains=1, steps=bench.SA_STEPS, seed=bench.RUN_SEED)
+    for c in [0, 1, 31, 4096, 40000, bench.CHAINS - 1, gid]:
+        assert oracle.sa_chain(pr, p, T0v, c)["E_best"] == cb[c], c
