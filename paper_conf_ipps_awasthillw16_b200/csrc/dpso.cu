@@ -43,7 +43,9 @@ struct DpArgs {
 
 template <int E, bool UCD>
 struct DpSmem {
-    static constexpr int BYTES = Chain<E, UCD>::BYTES + 128;  // + 32-word membership bitmap
+    static constexpr int NP = Chain<E, UCD>::NP;
+    // chain + 32-word membership bitmap + the two donor sequences (personal / swarm best)
+    static constexpr int BYTES = Chain<E, UCD>::BYTES + 128 + 2 * NP * 2;
 };
 
 __device__ __forceinline__ uint32_t lanemask_lt(int lane) { return (1u << lane) - 1u; }
@@ -60,7 +62,7 @@ __device__ __forceinline__ void build_bitmap(uint32_t* bm, const uint16_t* ids, 
     __syncwarp();
 }
 
-// Writes the jobs of `donor` (global, n entries) that are not in the bitmap, in donor order, to
+// Writes the jobs of `donor` (shared, n entries) that are not in the bitmap, in donor order, to
 // the positions produced by `dst(idx)` for idx = 0, 1, ...
 template <class Dst>
 __device__ __forceinline__ void compact_from(uint16_t* ids, const uint32_t* bm,
@@ -159,6 +161,8 @@ __global__ void __launch_bounds__(kDpThreads) dpso_iter_kernel(DpArgs a, int64_t
     uint8_t* wbase = smem + (size_t)wib * DpSmem<E, UCD>::BYTES;
     const C ch{wbase};
     uint32_t* bm = reinterpret_cast<uint32_t*>(wbase + C::BYTES);
+    int16_t* dpb = reinterpret_cast<int16_t*>(wbase + C::BYTES + 128);
+    int16_t* dg = dpb + C::NP;
     uint16_t* ids = ch.id();
     const int n = a.n;
     const int cur = (int)(t & 1), nxt = cur ^ 1;
@@ -168,7 +172,22 @@ __global__ void __launch_bounds__(kDpThreads) dpso_iter_kernel(DpArgs a, int64_t
     unsigned long long wkey = ULLONG_MAX;
     for (int64_t i = (int64_t)blockIdx.x * kDpWarps + wib; i < a.particles; i += total) {
         const uint64_t gid = a.offset + (uint64_t)i;
-        copy_in<E, UCD>(ids, a.pos + (size_t)i * a.np, lane);
+        // the position and both donors (personal best, swarm best) to shared memory in one batch
+        // of independent 16-byte loads, so the crossovers below never wait on global memory
+        {
+            constexpr int NP = C::NP;
+            const int16_t* gp = a.pos + (size_t)i * a.np;
+            const int16_t* gb = a.pb + (size_t)i * a.np;
+            for (int o = lane * 8; o < NP; o += 256) {
+                const int4 x = *reinterpret_cast<const int4*>(gp + o);
+                const int4 y = *reinterpret_cast<const int4*>(gb + o);
+                const int4 z = *reinterpret_cast<const int4*>(g + o);
+                *reinterpret_cast<int4*>(ids + o) = x;
+                *reinterpret_cast<int4*>(dpb + o) = y;
+                *reinterpret_cast<int4*>(dg + o) = z;
+            }
+            __syncwarp();
+        }
         // random words of (t, particle): lane 0 -> block 0, lane 1 -> block 1
         const uint4 wv = rng_block(a.seed, (uint32_t)t, gid, kTagDpso, (uint32_t)(lane & 1));
         const uint32_t a0 = __shfl_sync(kFull, wv.x, 0), a1 = __shfl_sync(kFull, wv.y, 0);
@@ -192,7 +211,7 @@ __global__ void __launch_bounds__(kDpThreads) dpso_iter_kernel(DpArgs a, int64_t
         if (__dmul_rn(__dadd_rn((double)a3, 0.5), u2) < a.c1) {
             const int c = 1 + (int)bnd(b0, (uint32_t)n - 1u);
             build_bitmap(bm, ids, 0, c - 1, lane);
-            compact_from(ids, bm, a.pb + (size_t)i * a.np, n, lane, [c](int idx) { return c + idx; });
+            compact_from(ids, bm, dpb, n, lane, [c](int idx) { return c + idx; });
         }
         // p(t+1) = c2 (+) F3(delta, g): two-point crossover with the swarm best
         if (__dmul_rn(__dadd_rn((double)b1, 0.5), u2) < a.c2) {
@@ -206,7 +225,7 @@ __global__ void __launch_bounds__(kDpThreads) dpso_iter_kernel(DpArgs a, int64_t
             }
             build_bitmap(bm, ids, q0, q1, lane);
             const int span = q1 - q0 + 1;
-            compact_from(ids, bm, g, n, lane,
+            compact_from(ids, bm, dg, n, lane,
                          [q0, span](int idx) { return idx < q0 ? idx : idx + span; });
         }
         // line 7: evaluate
