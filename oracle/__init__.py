@@ -53,7 +53,8 @@ class Walk(C.Structure):
 class SAParams(C.Structure):
     _fields_ = [("problem", C.c_int32), ("chains", C.c_int64), ("steps", C.c_int64),
                 ("mu", C.c_double), ("pert", C.c_int32), ("move", C.c_int32),
-                ("seed", C.c_uint64), ("chain_offset", C.c_uint64)]
+                ("seed", C.c_uint64), ("chain_offset", C.c_uint64), ("init", C.c_void_p),
+                ("init_ld", C.c_int64)]
 
 
 class DPSOParams(C.Structure):
@@ -214,8 +215,16 @@ def t0(prob: Problem, problem: int, seed: int, samples: int = 5000) -> float:
 
 
 def sa_params(problem=CDD, chains=1, steps=1000, mu=0.88, pert=4, move=MOVE_PERT_FY, seed=0,
-              chain_offset=0) -> SAParams:
-    return SAParams(problem, chains, steps, mu, pert, move, seed, chain_offset)
+              chain_offset=0, init=None) -> SAParams:
+    """init: None (random initial sequences), an int16 [n] array (every chain) or [chains, n]
+    (row c for chain c).  The array is kept alive on the returned struct."""
+    p = SAParams(problem, chains, steps, mu, pert, move, seed, chain_offset, None, 0)
+    if init is not None:
+        arr = np.ascontiguousarray(init, dtype=np.int16)
+        p._init = arr
+        p.init = arr.ctypes.data
+        p.init_ld = arr.shape[1] if arr.ndim == 2 else 0
+    return p
 
 
 def sa_chain(prob: Problem, p: SAParams, T0: float, g: int, trace: bool = False):

@@ -89,6 +89,11 @@ typedef struct {
     int32_t  move;          /* OR_MOVE_*                                  */
     uint64_t seed;
     uint64_t chain_offset;  /* global id of local chain 0                 */
+    /* Initial sequences ("the initial job sequences are copied to the GPU"): NULL = the
+     * chain's own random sequence (R13); else chain c = g - chain_offset starts from
+     * init + c * init_ld (init_ld = 0: every chain from the same sequence). */
+    const int16_t *init;
+    int64_t  init_ld;
 } or_sa_params;
 
 /* The neighbour move of SA step k of chain g: Pert distinct positions q[0..P-1] (ascending),

@@ -201,6 +201,24 @@ def test_sa_n10_reaches_the_nfact_optimum():
     assert r["E_best"] == z_opt
 
 
+def test_sa_initial_sequences():
+    # initial sequences copied to the device.  Giving each chain its own random sequence
+    # explicitly reproduces the default run; zero steps return the given sequence
+    inst, pr, p = _sa(n=30, steps=200, seed=6, chains=5, chain_offset=11)
+    T0 = oracle.t0(pr, oracle.CDD, 6, 300)
+    rows = np.stack([oracle.perm_fy(30, 6, oracle.TAG_SA_INIT, 11 + c) for c in range(5)])
+    a = oracle.sa_run(pr, p, T0, chain_best=True)
+    b = oracle.sa_run(pr, oracle.sa_params(chains=5, steps=200, seed=6, chain_offset=11, init=rows),
+                      T0, chain_best=True)
+    assert np.array_equal(a["chain_best"], b["chain_best"]) and np.array_equal(a["best"], b["best"])
+    v = np.argsort(inst.P / inst.alpha).astype(np.int16)
+    z = oracle.cdd_eval(pr, v)
+    r = oracle.sa_chain(pr, oracle.sa_params(chains=1, steps=0, seed=6, init=v), T0, 0)
+    assert r["E_best"] == z and np.array_equal(r["best"], v)
+    r = oracle.sa_chain(pr, oracle.sa_params(chains=1, steps=300, seed=6, init=v), T0, 0)
+    assert r["E_best"] <= z
+
+
 # ---------------------------------------------------------------------- synchronous SA (F2)
 def test_sa_sync_single_chain_unit_length_is_the_async_chain():
     # chains = 1, M = 1: level j is one move at T0*mu^j from the previous final state with the
