@@ -14,6 +14,8 @@
 #include <cuda_runtime.h>
 
 #include <cstdint>
+#include <cstdio>
+#include <cstdlib>
 
 #include "device_common.cuh"
 #include "internal.h"
@@ -21,8 +23,6 @@
 namespace cdd {
 namespace {
 
-constexpr int kE2Warps = 16;             // one 512-thread CTA per SM
-constexpr int kE2Threads = kE2Warps * 32;
 // Table copies KC: lane L reads copy L % KC; 16 copies (2-way-at-worst bank conflicts between
 // lanes L and L+16) when shared memory allows, else 8 (4 lanes per copy, ~2.9 wavefronts/gather).
 constexpr int kE2MaxSmem = 227 * 1024;
@@ -43,6 +43,19 @@ __host__ __device__ inline E2Layout e2_layout(uint32_t sbase, uint32_t tbytes, u
 __device__ __forceinline__ uint32_t lds32(uint32_t addr) {
     uint32_t v;
     asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(addr));
+    return v;
+}
+
+// Table gather: with TOFF != 0 the table sits at the start of the dynamic window (shared address
+// TOFF, the probed base) and the base rides in the load's immediate offset, so the table need not
+// be aligned to its size (room for 32 conflict-free copies at n = 1000).
+template <uint32_t TOFF>
+__device__ __forceinline__ uint32_t ldtab(uint32_t addr) {
+    uint32_t v;
+    if constexpr (TOFF == 0)
+        asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(addr));
+    else
+        asm volatile("ld.shared.u32 %0, [%1+%2];" : "=r"(v) : "r"(addr), "n"(TOFF));
     return v;
 }
 
@@ -78,8 +91,8 @@ struct E2 {
 };
 
 // One group of 32/G sequences per warp and stage.
-template <int G, int E>
-__global__ void __launch_bounds__(kE2Threads, 1) eval2_cdd_kernel(
+template <int G, int E, int W, uint32_t TOFF, bool TAIL>
+__global__ void __launch_bounds__(W * 32, 1) eval2_cdd_kernel(
     const uint16_t* __restrict__ tab_ab16, const uint8_t* __restrict__ tab_p, int n, int npow2,
     int kc_log2, int32_t d, const int16_t* __restrict__ perms, int64_t ld, int64_t batch,
     int64_t* __restrict__ out, int* __restrict__ err) {
@@ -91,8 +104,9 @@ __global__ void __launch_bounds__(kE2Threads, 1) eval2_cdd_kernel(
     const int KC = 1 << kc_log2;
     const uint32_t sbase = (uint32_t)__cvta_generic_to_shared(smem);
     const uint32_t tbytes = (uint32_t)npow2 * 4u * (uint32_t)KC;
-    const E2Layout Ly = e2_layout(sbase, tbytes, 2u * X::STAGE, kE2Warps);
-    const uint32_t tab = sbase + Ly.tab_off;
+    const E2Layout Ly = TOFF ? E2Layout{0u, 0u, tbytes + (uint32_t)W * 2u * X::STAGE}
+                             : e2_layout(sbase, tbytes, 2u * X::STAGE, W);
+    const uint32_t tab = TOFF ? 0u : sbase + Ly.tab_off;
     const uint32_t stage0 = sbase + ((uint32_t)warp < Ly.nb ? (uint32_t)warp * 2u * X::STAGE
                                                               : Ly.tab_off + tbytes + ((uint32_t)warp - Ly.nb) * 2u * X::STAGE);
     uint32_t* s_tab = reinterpret_cast<uint32_t*>(smem + Ly.tab_off);
@@ -106,8 +120,9 @@ __global__ void __launch_bounds__(kE2Threads, 1) eval2_cdd_kernel(
     const uint32_t tabc = tab | (uint32_t)((lane & (KC - 1)) * 4);
 
     const int cpr = (n + 7) / 8;  // 16-byte chunks of real ids per sequence (ld % 8 == 0)
+    const uint32_t S = (uint32_t)npow2 - 1u;  // sentinel id: >= n, zero record
     const int64_t ngroups = (batch + CPW - 1) / CPW;
-    const int64_t gstep = (int64_t)gridDim.x * kE2Warps;
+    const int64_t gstep = (int64_t)gridDim.x * W;
     // this lane copies chunks cg = lane + 32 t of every sequence of a group (its stage slot
     // depends on the group only through nothing: the offsets are loop invariants)
     auto issue = [&](int64_t rg, int st) {
@@ -128,13 +143,32 @@ __global__ void __launch_bounds__(kE2Threads, 1) eval2_cdd_kernel(
         cp_async_commit();
     };
 
-    const int64_t rg0 = (int64_t)blockIdx.x * kE2Warps + warp;
+    // Slots past the sequence's last real chunk are never copied: fill them once with the sentinel
+    // id S = npow2 - 1 (>= n, a zero record); ids there are excluded from the validity check.
+    {
+        const uint4 s4 = make_uint4(S * 0x10001u, S * 0x10001u, S * 0x10001u, S * 0x10001u);
+        for (int st = 0; st < 2; ++st)
+#pragma unroll
+            for (int r = 0; r < CPW; ++r)
+                for (int cg = cpr + lane; cg < G * CPS; cg += 32) {
+                    const int seg = cg / CPS, c = cg % CPS;
+                    const uint32_t slot = (uint32_t)(seg * CPS) + ((uint32_t)c ^ X::sw(r * G + seg));
+                    const uint32_t a = stage0 + (uint32_t)(st * X::STAGE + r * X::ROWB) + 16u * slot;
+                    asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};" ::"r"(a), "r"(s4.x), "r"(s4.y),
+                                 "r"(s4.z), "r"(s4.w) : "memory");
+                }
+        __syncwarp();
+    }
+    const int64_t rg0 = (int64_t)blockIdx.x * W + warp;
     issue(rg0, 0);
     issue(rg0 + gstep, 1);
     uint32_t vmax = 0;
     bool bad = false;
-    const uint32_t s2 = (uint32_t)n * 0x10001u;  // two sentinel ids (zero records)
     const uint32_t sw_own = X::sw(grp * G + l);
+    const int kown = min(E, max(0, n - l * E));  // positions of own segment before n
+    const int nfull_lane = kown / 8;
+    const int cstr = (kown % 8) ? kown / 8 : -1;  // chunk straddling n (n % 8 != 0 only)
+    const int kstr = kown % 8;  // real ids in that chunk
     int it = 0;
     for (int64_t rg = rg0; rg < ngroups; rg += gstep, ++it) {
         const int st = it & 1;
@@ -143,35 +177,41 @@ __global__ void __launch_bounds__(kE2Threads, 1) eval2_cdd_kernel(
         const uint32_t srow = stage0 + (uint32_t)(st * X::STAGE) + (uint32_t)(grp * X::ROWB);
         const int64_t row = rg * CPW + grp;
         const bool rv = row < batch;
-        const int kmax = rv ? min(E, max(0, n - l * E)) : 0;  // valid positions in own segment
         // ---- gather: 16-bit alpha|beta<<8 pairs and p bytes, lane totals
         uint32_t abp[E / 2], pw[E / 4];
         uint32_t tA = 0, tB = 0, tP = 0;
         const uint32_t seg_addr = srow + (uint32_t)(l * CPS * 16);
-#pragma unroll
-        for (int c = 0; c < CPS; ++c) {
-            uint4 q = lds128(seg_addr + (((uint32_t)c ^ sw_own) << 4));
-            if (8 * c + 8 <= kmax) {
-                vmax = __vmaxu2(vmax, __vmaxu2(__vmaxu2(q.x, q.y), __vmaxu2(q.z, q.w)));
-            } else if (8 * c >= kmax) {  // wholly past n (or an idle row): zero records
-                q = make_uint4(s2, s2, s2, s2);
-            } else {  // the chunk straddling n (n % 8 != 0): check real ids, sentinel the rest
+        const int nfull = rv ? nfull_lane : 0;  // chunks of own segment wholly before n
+        if constexpr (TAIL) {
+            // n % 8 != 0: the lane owning the chunk that straddles n checks its real ids and
+            // overwrites the rest (the caller's padding) with the sentinel, in place
+            if (cstr >= 0) {
+                const uint32_t a = seg_addr + (((uint32_t)cstr ^ sw_own) << 4);
+                const uint4 q = lds128(a);
                 uint32_t ws[4] = {q.x, q.y, q.z, q.w};
 #pragma unroll
                 for (int j = 0; j < 4; ++j) {
                     uint32_t lo = ws[j] & 0xffffu, hi = ws[j] >> 16;
-                    if (8 * c + 2 * j < kmax) bad |= lo >= (uint32_t)n; else lo = s2 & 0xffffu;
-                    if (8 * c + 2 * j + 1 < kmax) bad |= hi >= (uint32_t)n; else hi = s2 & 0xffffu;
+                    if (2 * j < kstr) bad |= rv && lo >= (uint32_t)n; else lo = S;
+                    if (2 * j + 1 < kstr) bad |= rv && hi >= (uint32_t)n; else hi = S;
                     ws[j] = lo | (hi << 16);
                 }
-                q = make_uint4(ws[0], ws[1], ws[2], ws[3]);
+                asm volatile("st.shared.v4.u32 [%0], {%1,%2,%3,%4};" ::"r"(a), "r"(ws[0]), "r"(ws[1]),
+                             "r"(ws[2]), "r"(ws[3]) : "memory");
             }
+            __syncwarp();
+        }
+#pragma unroll
+        for (int c = 0; c < CPS; ++c) {
+            uint4 q = lds128(seg_addr + (((uint32_t)c ^ sw_own) << 4));
+            // chunks wholly past n hold the sentinel (written once, never copied over)
+            if (c < nfull) vmax = __vimax3_u16x2(__vimax3_u16x2(vmax, q.x, q.y), q.z, q.w);
             const uint32_t wv[4] = {q.x, q.y, q.z, q.w};
             uint32_t r[8];
 #pragma unroll
             for (int j = 0; j < 4; ++j) {
-                r[2 * j] = lds32(((wv[j] << SH) & amask) | tabc);
-                r[2 * j + 1] = lds32(((wv[j] >> (16 - SH)) & amask) | tabc);
+                r[2 * j] = ldtab<TOFF>(((wv[j] << SH) & amask) | tabc);
+                r[2 * j + 1] = ldtab<TOFF>(((wv[j] >> (16 - SH)) & amask) | tabc);
             }
 #pragma unroll
             for (int j = 0; j < 4; ++j) {
@@ -238,7 +278,7 @@ __global__ void __launch_bounds__(kE2Threads, 1) eval2_cdd_kernel(
 #pragma unroll
         for (int i = 0; i < SPR; ++i) {
             const uint32_t id = (i & 1) ? (idw[i >> 1] >> 16) : (idw[i >> 1] & 0xffffu);
-            const uint32_t rec = (rv && kb + i < n) ? lds32(((id << SH) & amask) | tabc) : 0u;
+            const uint32_t rec = (rv && kb + i < n) ? ldtab<TOFF>(((id << SH) & amask) | tabc) : 0u;
             // p | (alpha + beta) << 16
             v[i] = __byte_perm(rec, 0u, 0x4442u) + (__dp4a(rec, 0x00000101u, 0u) << 16);
             lsum += v[i];
@@ -285,33 +325,44 @@ __global__ void __launch_bounds__(kE2Threads, 1) eval2_cdd_kernel(
     if (bad || (vmax & 0xffffu) >= (uint32_t)n || (vmax >> 16) >= (uint32_t)n) atomicOr(err, 1);
 }
 
-template <int G, int E>
+// kc_log2 = log2 of the table copies (5: conflict free, 4, 3); W warps per CTA; TOFF != 0 puts the
+// table at the window start (needs the probed base to equal TOFF).  cudaErrorNotSupported if the
+// layout does not fit.
+template <int G, int E, int W, uint32_t TOFF>
 cudaError_t launch2(const Instance& I, const int16_t* perms, int64_t ld, int64_t batch,
-                    int64_t* out, cudaStream_t s) {
+                    int64_t* out, cudaStream_t s, int kc_log2) {
     using X = E2<G, E>;
+    if (TOFF != 0 && I.smem_base != TOFF) return cudaErrorNotSupported;
     int npow2 = 1;
     while (npow2 <= I.n) npow2 <<= 1;
-    int kc_log2 = 4;
-    E2Layout Ly = e2_layout(I.smem_base, (uint32_t)npow2 * 4u << kc_log2, 2u * X::STAGE, kE2Warps);
-    if (Ly.total > (uint32_t)kE2MaxSmem) {
-        kc_log2 = 3;
-        Ly = e2_layout(I.smem_base, (uint32_t)npow2 * 4u << kc_log2, 2u * X::STAGE, kE2Warps);
-    }
-    if (Ly.total > (uint32_t)kE2MaxSmem) return cudaErrorNotSupported;
-    const size_t smem = Ly.total;
-    auto kern = eval2_cdd_kernel<G, E>;
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    const uint32_t tbytes = (uint32_t)npow2 * 4u << kc_log2;
+    const uint32_t total = TOFF ? tbytes + (uint32_t)W * 2u * X::STAGE
+                                : e2_layout(I.smem_base, tbytes, 2u * X::STAGE, W).total;
+    if (total > (uint32_t)kE2MaxSmem) return cudaErrorNotSupported;
+    auto kern = (I.n % 8) ? eval2_cdd_kernel<G, E, W, TOFF, true> : eval2_cdd_kernel<G, E, W, TOFF, false>;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)total);
     if (e != cudaSuccess) return e;
     int sms = 148;
     e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, I.device);
     if (e != cudaSuccess) return e;
     const int64_t groups = (batch + X::CPW - 1) / X::CPW;
-    int64_t blocks = (groups + kE2Warps - 1) / kE2Warps;
+    int64_t blocks = (groups + W - 1) / W;
     if (blocks > sms) blocks = sms;
     if (blocks < 1) blocks = 1;
-    kern<<<(unsigned)blocks, kE2Threads, smem, s>>>(I.tab_ab16, I.tab_p, I.n, npow2, kc_log2, I.d_eff,
-                                                    perms, ld, batch, out, I.err);
+    kern<<<(unsigned)blocks, W * 32, total, s>>>(I.tab_ab16, I.tab_p, I.n, npow2, kc_log2, I.d_eff,
+                                                 perms, ld, batch, out, I.err);
     return cudaGetLastError();
+}
+
+// Most copies that fit (32, 16, 8), W = 16 warps, table aligned to its size.
+template <int G, int E>
+cudaError_t launch2_auto(const Instance& I, const int16_t* perms, int64_t ld, int64_t batch,
+                         int64_t* out, cudaStream_t s) {
+    for (int kc = 5; kc >= 3; --kc) {
+        const cudaError_t e = launch2<G, E, 16, 0>(I, perms, ld, batch, out, s, kc);
+        if (e != cudaErrorNotSupported) return e;
+    }
+    return cudaErrorNotSupported;
 }
 
 __global__ void smem_base_probe(uint32_t* out) {
@@ -338,11 +389,21 @@ cudaError_t launch_eval2_cdd(const Instance& I, const int16_t* perms, int64_t ld
         return cudaErrorNotSupported;
     const int n = I.n;
     if (n <= 16) return cudaErrorNotSupported;  // one-warp-per-many-rows kernel of eval.cu is faster
-    if (n <= 64) return launch2<4, 16>(I, perms, ld, batch, out, s);
-    if (n <= 128) return launch2<4, 32>(I, perms, ld, batch, out, s);
-    if (n <= 256) return launch2<8, 32>(I, perms, ld, batch, out, s);
-    if (n <= 512) return launch2<8, 64>(I, perms, ld, batch, out, s);
-    return launch2<16, 64>(I, perms, ld, batch, out, s);
+    if (const char* cfg = getenv("CDD_EVAL2_CFG"); cfg && n > 512) {  // layout experiments
+        int w = 16, flat = 0, kc = 4;
+        sscanf(cfg, "%d:%d:%d", &w, &flat, &kc);
+        if (w == 8) return flat ? launch2<16, 64, 8, 1024>(I, perms, ld, batch, out, s, kc)
+                                : launch2<16, 64, 8, 0>(I, perms, ld, batch, out, s, kc);
+        if (w == 12) return flat ? launch2<16, 64, 12, 1024>(I, perms, ld, batch, out, s, kc)
+                                 : launch2<16, 64, 12, 0>(I, perms, ld, batch, out, s, kc);
+        return flat ? launch2<16, 64, 16, 1024>(I, perms, ld, batch, out, s, kc)
+                    : launch2<16, 64, 16, 0>(I, perms, ld, batch, out, s, kc);
+    }
+    if (n <= 64) return launch2_auto<4, 16>(I, perms, ld, batch, out, s);
+    if (n <= 128) return launch2_auto<4, 32>(I, perms, ld, batch, out, s);
+    if (n <= 256) return launch2_auto<8, 32>(I, perms, ld, batch, out, s);
+    if (n <= 512) return launch2_auto<8, 64>(I, perms, ld, batch, out, s);
+    return launch2_auto<16, 64>(I, perms, ld, batch, out, s);
 }
 
 }  // namespace cdd
