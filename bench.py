@@ -434,10 +434,14 @@ def bench_eval(lib, g, dev, stream, peaks, batch=1 << 20, reps=20):
     bytes_per = batch * (2 * N_JOBS + 8)
     gbs = bytes_per / (ms / 1000) / 1e9
     hbm = float(peaks.get("hbm_gbs", 6454.0))
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "eval_kernel_dram_bytes.json")
+    if os.path.exists(tp):
+        traffic = json.load(open(tp)).get("dram_bytes_per_launch")
     return {"workload": "cdd_eval_batch, CDD n=1000 h=0.4, 2^20 random sequences (2 GiB, alternating pools > L2)",
             "evals_per_s": batch / (ms / 1000), "ms_per_launch": ms,
             "roofline": {"bound": "hbm", "achieved": gbs, "peak": hbm, "unit": "GB/s",
-                         "frac": gbs / hbm, "traffic": None,
+                         "frac": gbs / hbm, "traffic": traffic, "bytes_per_launch": bytes_per,
                          "algorithmic_bytes_per_eval": 2 * N_JOBS + 8}}
 
 

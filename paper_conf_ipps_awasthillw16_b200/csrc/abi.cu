@@ -534,7 +534,7 @@ int dpso_run(cdd_instance* I, const dpso_params* p, void* ws, size_t ws_bytes, v
     DeviceGuard g(I->device);
     cudaStream_t s = as_stream(stream);
     cudaError_t e = cdd::dpso_begin(*I, L, ws, s);
-    for (int64_t t = 0; e == cudaSuccess && t < L.iters; ++t) e = cdd::dpso_iterate(*I, L, ws, t, s);
+    if (e == cudaSuccess) e = cdd::dpso_iterate(*I, L, ws, 0, L.iters, s);
     if (e == cudaSuccess) e = cdd::dpso_end(*I, L, ws, s);
     if (e != cudaSuccess) return cuda_fail(e, "dpso_run");
     I->has_best = true;
@@ -557,7 +557,7 @@ int dpso_iterate(cdd_instance* I, const dpso_params* p, void* ws, size_t ws_byte
     if (rc != CDD_OK) return rc;
     if (t < 0 || t >= L.iters) return fail(CDD_EINVAL, "t must be in [0, iters)");
     DeviceGuard g(I->device);
-    cudaError_t e = cdd::dpso_iterate(*I, L, ws, t, as_stream(stream));
+    cudaError_t e = cdd::dpso_iterate(*I, L, ws, t, t + 1, as_stream(stream));
     return e == cudaSuccess ? CDD_OK : cuda_fail(e, "dpso_iterate");
 }
 

@@ -7,8 +7,11 @@
 // finish copies the winner's personal best into the double-buffered swarm-best sequence).  The
 // kernel boundary is the swarm-wide barrier Alg. 2 needs between lines 5 and 6.
 //
-// The crossovers use a job-membership bitmap in shared memory and ballot/popc stream compaction
-// over the donor sequence (personal best for F2, swarm best for F3).
+// The crossovers keep the position of every job (inv) next to the sequence: a donor job is missing
+// from the kept part iff its position lies outside it, so the donor row (read from global memory
+// with 16-byte loads issued up front) is filtered with one shared-memory lookup per job, and the
+// kept jobs are ranked by a warp scan of per-lane counts.  The instance tables are staged in
+// shared memory once per CTA.
 #include <cuda_runtime.h>
 
 #include <climits>
@@ -44,49 +47,13 @@ struct DpArgs {
 template <int E, bool UCD>
 struct DpSmem {
     static constexpr int NP = Chain<E, UCD>::NP;
-    // chain + 32-word membership bitmap + the two donor sequences (personal / swarm best)
-    static constexpr int BYTES = Chain<E, UCD>::BYTES + 128 + 2 * NP * 2;
+    // per warp: the chain only (in the iteration kernel the position-of-job array lives in the
+    // record area, which is rebuilt after the crossovers) ...
+    static constexpr int BYTES = Chain<E, UCD>::BYTES;
+    static constexpr int WARP = BYTES;
+    // ... and, per CTA, the instance tables by job id: ab u32, p (or M) u8 [, X u8, gamma u16]
+    static constexpr int TAB = NP * (UCD ? 8 : 5);
 };
-
-__device__ __forceinline__ uint32_t lanemask_lt(int lane) { return (1u << lane) - 1u; }
-
-// Membership bitmap of ids[lo..hi] (inclusive).
-__device__ __forceinline__ void build_bitmap(uint32_t* bm, const uint16_t* ids, int lo, int hi,
-                                             int lane) {
-    bm[lane] = 0u;
-    __syncwarp();
-    for (int k = lo + lane; k <= hi; k += 32) {
-        const int j = ids[k];
-        atomicOr(&bm[j >> 5], 1u << (j & 31));
-    }
-    __syncwarp();
-}
-
-// Writes the jobs of `donor` (shared, n entries) that are not in the bitmap, in donor order, to
-// the positions produced by `dst(idx)` for idx = 0, 1, ...
-template <class Dst>
-__device__ __forceinline__ void compact_from(uint16_t* ids, const uint32_t* bm,
-                                             const int16_t* __restrict__ donor, int n, int lane,
-                                             Dst&& dst) {
-    int out = 0;
-    for (int base = 0; base < n; base += 32) {
-        const int k = base + lane;
-        const int job = k < n ? (int)donor[k] : 0;
-        const bool keep = k < n && !((bm[job >> 5] >> (job & 31)) & 1u);
-        const uint32_t m = __ballot_sync(kFull, keep);
-        if (keep) ids[dst(out + __popc(m & lanemask_lt(lane)))] = (uint16_t)job;
-        out += __popc(m);
-    }
-    __syncwarp();
-}
-
-template <int E, bool UCD>
-__device__ __forceinline__ void copy_in(uint16_t* ids, const int16_t* src, int lane) {
-    constexpr int NP = Chain<E, UCD>::NP;
-    for (int o = lane * 8; o < NP; o += 256)
-        *reinterpret_cast<int4*>(ids + o) = *reinterpret_cast<const int4*>(src + o);
-    __syncwarp();
-}
 
 template <int E, bool UCD>
 __device__ __forceinline__ void copy_out(int16_t* dst, const uint16_t* ids, int lane) {
@@ -140,6 +107,10 @@ __global__ void __launch_bounds__(kDpThreads) dpso_init_kernel(DpArgs a) {
     for (int64_t i = (int64_t)blockIdx.x * kDpWarps + wib; i < a.particles; i += total) {
         const uint64_t gid = a.offset + (uint64_t)i;
         chain_fy_init<E, UCD>(ch, a.n, a.seed, kTagDpsoInit, gid, lane);
+        // positions past n carry the sentinel id NP - 1 (>= n: a zero record in the iteration
+        // kernel's table); the crossovers never move them
+        for (int k = a.n + lane; k < C::NP; k += 32) ch.id()[k] = (uint16_t)(C::NP - 1);
+        __syncwarp();
         chain_build<E, UCD>(ch, a.T, a.n, lane);
         const int32_t z = chain_eval<E, UCD>(ch, lane, a.n, a.d);
         copy_out<E, UCD>(a.pos + (size_t)i * a.np, ch.id(), lane);
@@ -152,39 +123,181 @@ __global__ void __launch_bounds__(kDpThreads) dpso_init_kernel(DpArgs a) {
     publish<E, UCD>(a, wkey, 0, 1, false);
 }
 
-// Lines 6-7 of iteration t, then lines 4-5 of iteration t+1.
+// Instance tables by job id, staged in shared memory once per CTA at `t`: ab u32 [NP], p (or M)
+// u8 [NP], UCDDCP: X u8 [NP], gamma u16 [NP].
 template <int E, bool UCD>
+struct DpTab {
+    static constexpr int NP = Chain<E, UCD>::NP;
+    const uint8_t* t;
+    __device__ __forceinline__ uint32_t ab(int j) const { return reinterpret_cast<const uint32_t*>(t)[j]; }
+    __device__ __forceinline__ uint8_t p(int j) const { return t[4 * NP + j]; }
+    __device__ __forceinline__ uint8_t x(int j) const { return t[5 * NP + j]; }
+    __device__ __forceinline__ uint16_t g(int j) const { return reinterpret_cast<const uint16_t*>(t + 6 * NP)[j]; }
+};
+
+template <int E, bool UCD>
+__device__ __forceinline__ void stage_tables(uint8_t* t, const ChainTables& T, int n, bool fast) {
+    constexpr int NP = Chain<E, UCD>::NP;
+    if (fast) {  // CDD with 8-bit alpha, beta: one record alpha | beta << 8 | p << 16, zero past n
+        for (int j = threadIdx.x; j < NP; j += blockDim.x)
+            reinterpret_cast<uint32_t*>(t)[j] =
+                j < n ? (uint32_t)__ldg(T.ab16 + j) | ((uint32_t)__ldg(T.p + j) << 16) : 0u;
+        return;
+    }
+    for (int j = threadIdx.x; j < n; j += blockDim.x) {
+        reinterpret_cast<uint32_t*>(t)[j] = __ldg(T.ab + j);
+        t[4 * NP + j] = __ldg(T.p + j);
+        if constexpr (UCD) {
+            t[5 * NP + j] = __ldg(T.x + j);
+            reinterpret_cast<uint16_t*>(t + 6 * NP)[j] = __ldg(T.g + j);
+        }
+    }
+}
+
+// Records of the sequence in id[] from the shared-memory tables (positions >= n: zero records).
+template <int E, bool UCD>
+__device__ __forceinline__ void chain_build_s(const Chain<E, UCD>& ch, const DpTab<E, UCD>& S, int n,
+                                              int lane) {
+    using C = Chain<E, UCD>;
+    const uint16_t* ids = ch.id();
+#pragma unroll 4
+    for (int k = lane; k < C::NP; k += 32) {
+        const bool v = k < n;
+        const int j = v ? ids[k] : 0;
+        ch.ab()[C::ab_w(k)] = v ? S.ab(j) : 0u;
+        ch.pb()[C::pb_b(k)] = v ? S.p(j) : (uint8_t)0;
+        if constexpr (UCD) {
+            ch.xb()[C::pb_b(k)] = v ? S.x(j) : (uint8_t)0;
+            ch.gh()[C::gh_h(k)] = v ? S.g(j) : (uint16_t)0;
+        }
+    }
+    __syncwarp();
+}
+
+// The same records from the packed table (CDD, E >= 8): lane l builds its own segment
+// [l*E, l*E+E) -- ids by 16-byte loads, one table load per position, the alpha|beta words and p
+// bytes assembled by PRMT and written with 16-byte stores.  Positions past n hold the sentinel id,
+// whose record is zero.
+template <int E>
+__device__ __forceinline__ void chain_build_fast(const Chain<E, false>& ch, const uint32_t* rtab, int lane) {
+    using C = Chain<E, false>;
+    static_assert(E >= 8, "16-byte segments");
+    const uint16_t* ids = ch.id() + lane * E;
+    uint32_t* abw = ch.ab() + lane * C::AB_STRIDE;
+    uint8_t* pb = ch.pb() + lane * C::PB_STRIDE;
+#pragma unroll
+    for (int v = 0; v < E / 8; ++v) {
+        const uint4 q = *reinterpret_cast<const uint4*>(ids + 8 * v);
+        const uint32_t w[4] = {q.x, q.y, q.z, q.w};
+        uint32_t r[8];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            r[2 * j] = rtab[w[j] & 0xffffu];
+            r[2 * j + 1] = rtab[w[j] >> 16];
+        }
+        uint32_t a[8];
+#pragma unroll
+        for (int j = 0; j < 8; ++j) a[j] = __byte_perm(r[j], 0u, 0x4140u);  // alpha | beta << 16
+        *reinterpret_cast<uint4*>(abw + 8 * v) = make_uint4(a[0], a[1], a[2], a[3]);
+        *reinterpret_cast<uint4*>(abw + 8 * v + 4) = make_uint4(a[4], a[5], a[6], a[7]);
+        const uint32_t p0 = __byte_perm(__byte_perm(r[0], r[1], 0x0062u), __byte_perm(r[2], r[3], 0x0062u), 0x5410u);
+        const uint32_t p1 = __byte_perm(__byte_perm(r[4], r[5], 0x0062u), __byte_perm(r[6], r[7], 0x0062u), 0x5410u);
+        *reinterpret_cast<uint2*>(pb + 8 * v) = make_uint2(p0, p1);
+    }
+    __syncwarp();
+}
+
+__device__ __forceinline__ uint32_t warp_excl_scan(uint32_t v, int lane, uint32_t* total) {
+    uint32_t x = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(kFull, x, o);
+        if (lane >= o) x += y;
+    }
+    *total = __shfl_sync(kFull, x, 31);
+    return x - v;
+}
+
+// Crossover fill: the jobs of `donor` (global row, n entries) for which keep(inv[job]) holds are
+// written, in donor order, to positions dst(0), dst(1), ... of ids[], and inv[] follows them.
+// The donor row is read with 16-byte loads issued up front (lane L holds donor positions
+// [8L + 256 r, 8L + 256 r + 8)); the rank of a kept job is a warp scan of per-lane counts.
+template <int E, class Keep, class Dst>
+__device__ __forceinline__ void fill_from(uint16_t* ids, uint16_t* inv, const int16_t* __restrict__ donor,
+                                          int n, int lane, Keep&& keep, Dst&& dst) {
+    constexpr int R = (32 * E + 255) / 256;  // 16-byte rounds per lane
+    uint4 q[R];
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+        const int o = 8 * lane + 256 * r;
+        q[r] = o < 32 * E ? __ldg(reinterpret_cast<const uint4*>(donor + o)) : make_uint4(0, 0, 0, 0);
+    }
+    uint32_t km[R];
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+        const uint32_t w[4] = {q[r].x, q[r].y, q[r].z, q[r].w};
+        uint32_t m = 0;
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+            const int k = 8 * lane + 256 * r + j;
+            const uint32_t job = (j & 1) ? (w[j >> 1] >> 16) : (w[j >> 1] & 0xffffu);
+            if (k < n && keep((int)inv[job])) m |= 1u << j;
+        }
+        km[r] = m;
+    }
+    __syncwarp();
+    int out = 0;
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+        uint32_t tot;
+        int idx = out + (int)warp_excl_scan((uint32_t)__popc(km[r]), lane, &tot);
+        out += (int)tot;
+        const uint32_t w[4] = {q[r].x, q[r].y, q[r].z, q[r].w};
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+            if ((km[r] >> j) & 1u) {
+                const uint32_t job = (j & 1) ? (w[j >> 1] >> 16) : (w[j >> 1] & 0xffffu);
+                const int pos = dst(idx++);
+                ids[pos] = (uint16_t)job;
+                inv[job] = (uint16_t)pos;
+            }
+        }
+    }
+    __syncwarp();
+}
+
+// Lines 6-7 of iteration t, then lines 4-5 of iteration t+1.
+template <int E, bool UCD, bool FAST>
 __global__ void __launch_bounds__(kDpThreads) dpso_iter_kernel(DpArgs a, int64_t t) {
     using C = Chain<E, UCD>;
+    constexpr int NP = C::NP;
     extern __shared__ __align__(16) uint8_t smem[];
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
-    uint8_t* wbase = smem + (size_t)wib * DpSmem<E, UCD>::BYTES;
-    const C ch{wbase};
-    uint32_t* bm = reinterpret_cast<uint32_t*>(wbase + C::BYTES);
-    int16_t* dpb = reinterpret_cast<int16_t*>(wbase + C::BYTES + 128);
-    int16_t* dg = dpb + C::NP;
+    stage_tables<E, UCD>(smem, a.T, a.n, FAST);
+    const DpTab<E, UCD> S{smem};
+    const C ch{smem + DpSmem<E, UCD>::TAB + (size_t)wib * DpSmem<E, UCD>::WARP};
     uint16_t* ids = ch.id();
+    uint16_t* inv = reinterpret_cast<uint16_t*>(ch.ab());  // position of each job (crossovers only)
     const int n = a.n;
     const int cur = (int)(t & 1), nxt = cur ^ 1;
     if (a.trace && blockIdx.x == 0 && threadIdx.x == 0) a.trace[t] = (int64_t)(a.gkey[cur] >> 32);
     const int16_t* g = a.gperm + (size_t)cur * a.np;
     const int64_t total = (int64_t)gridDim.x * kDpWarps;
     unsigned long long wkey = ULLONG_MAX;
+    __syncthreads();
     for (int64_t i = (int64_t)blockIdx.x * kDpWarps + wib; i < a.particles; i += total) {
         const uint64_t gid = a.offset + (uint64_t)i;
-        // the position and both donors (personal best, swarm best) to shared memory in one batch
-        // of independent 16-byte loads, so the crossovers below never wait on global memory
+        // the position to shared memory (16-byte loads) and the position of every job
         {
-            constexpr int NP = C::NP;
             const int16_t* gp = a.pos + (size_t)i * a.np;
-            const int16_t* gb = a.pb + (size_t)i * a.np;
+#pragma unroll
             for (int o = lane * 8; o < NP; o += 256) {
-                const int4 x = *reinterpret_cast<const int4*>(gp + o);
-                const int4 y = *reinterpret_cast<const int4*>(gb + o);
-                const int4 z = *reinterpret_cast<const int4*>(g + o);
-                *reinterpret_cast<int4*>(ids + o) = x;
-                *reinterpret_cast<int4*>(dpb + o) = y;
-                *reinterpret_cast<int4*>(dg + o) = z;
+                const uint4 x = __ldg(reinterpret_cast<const uint4*>(gp + o));
+                *reinterpret_cast<uint4*>(ids + o) = x;
+                const uint32_t w[4] = {x.x, x.y, x.z, x.w};
+#pragma unroll  // (positions past n hold the sentinel NP - 1, whose entry is never read)
+                for (int j = 0; j < 8; ++j)
+                    inv[(j & 1) ? (w[j >> 1] >> 16) : (w[j >> 1] & 0xffffu)] = (uint16_t)(o + j);
             }
             __syncwarp();
         }
@@ -201,19 +314,23 @@ __global__ void __launch_bounds__(kDpThreads) dpso_iter_kernel(DpArgs a, int64_t
             int qb = (int)bnd(a2, (uint32_t)n);
             if (qb == pa) qb = n - 1;
             if (lane == 0) {
-                const uint16_t x = ids[pa];
-                ids[pa] = ids[qb];
+                const uint16_t x = ids[pa], y = ids[qb];
+                ids[pa] = y;
                 ids[qb] = x;
+                inv[y] = (uint16_t)pa;
+                inv[x] = (uint16_t)qb;
             }
             __syncwarp();
         }
-        // delta = c1 (+) F2(lambda, p^b): one-point crossover with the personal best
+        // delta = c1 (+) F2(lambda, p^b): one-point crossover with the personal best -- lambda's
+        // first c jobs stay, the others follow in personal-best order
         if (__dmul_rn(__dadd_rn((double)a3, 0.5), u2) < a.c1) {
             const int c = 1 + (int)bnd(b0, (uint32_t)n - 1u);
-            build_bitmap(bm, ids, 0, c - 1, lane);
-            compact_from(ids, bm, dpb, n, lane, [c](int idx) { return c + idx; });
+            fill_from<E>(ids, inv, a.pb + (size_t)i * a.np, n, lane, [c](int at) { return at >= c; },
+                         [c](int idx) { return c + idx; });
         }
-        // p(t+1) = c2 (+) F3(delta, g): two-point crossover with the swarm best
+        // p(t+1) = c2 (+) F3(delta, g): two-point crossover with the swarm best -- delta[q0..q1]
+        // stays, the other positions take the remaining jobs in swarm-best order
         if (__dmul_rn(__dadd_rn((double)b1, 0.5), u2) < a.c2) {
             int q0 = (int)bnd(b2, (uint32_t)n - 1u);
             int q1 = (int)bnd(b3, (uint32_t)n);
@@ -223,13 +340,15 @@ __global__ void __launch_bounds__(kDpThreads) dpso_iter_kernel(DpArgs a, int64_t
                 q0 = q1;
                 q1 = x;
             }
-            build_bitmap(bm, ids, q0, q1, lane);
             const int span = q1 - q0 + 1;
-            compact_from(ids, bm, dg, n, lane,
+            fill_from<E>(ids, inv, g, n, lane, [q0, q1](int at) { return at < q0 || at > q1; },
                          [q0, span](int idx) { return idx < q0 ? idx : idx + span; });
         }
         // line 7: evaluate
-        chain_build<E, UCD>(ch, a.T, n, lane);
+        if constexpr (FAST)
+            chain_build_fast<E>(ch, reinterpret_cast<const uint32_t*>(smem), lane);
+        else
+            chain_build_s<E, UCD>(ch, S, n, lane);
         const int32_t z = chain_eval<E, UCD>(ch, lane, n, a.d);
         copy_out<E, UCD>(a.pos + (size_t)i * a.np, ids, lane);
         // line 4 (iteration t+1): personal best
@@ -276,7 +395,7 @@ DpWs dp_layout(int np, int64_t N) {
 
 ChainTables dp_tables(const Instance& I, bool ucd) {
     return ucd ? ChainTables{I.tab_ab, I.tab_m, I.tab_x, I.tab_g}
-               : ChainTables{I.tab_ab, I.tab_p, nullptr, nullptr};
+               : ChainTables{I.tab_ab, I.tab_p, nullptr, nullptr, I.ab16_ok ? I.tab_ab16 : nullptr};
 }
 
 template <int E>
@@ -330,13 +449,22 @@ cudaError_t begin_e(Instance& I, const DpsoLaunch& p, void* ws, cudaStream_t s) 
     return cudaGetLastError();
 }
 
+// Iterations t0..t1-1 (the grid is sized once: the attribute queries cost more host time than a
+// launch).
 template <int E, bool UCD>
-cudaError_t iter_e(Instance& I, const DpsoLaunch& p, void* ws, int64_t t, cudaStream_t s) {
+cudaError_t iter_e(Instance& I, const DpsoLaunch& p, void* ws, int64_t t0, int64_t t1, cudaStream_t s) {
     const DpArgs a = make_args<E>(I, p, ws);
-    const size_t smem = kDpWarps * (size_t)DpSmem<E, UCD>::BYTES;
-    const int blocks = grid_for(I, dpso_iter_kernel<E, UCD>, smem, p.particles);
-    dpso_iter_kernel<E, UCD><<<blocks, kDpThreads, smem, s>>>(a, t);
-    return cudaGetLastError();
+    const size_t smem = DpSmem<E, UCD>::TAB + kDpWarps * (size_t)DpSmem<E, UCD>::WARP;
+    constexpr bool can_fast = !UCD && E >= 8;
+    const bool fast = can_fast && I.ab16_ok;
+    auto kern = fast ? dpso_iter_kernel<E, UCD, can_fast> : dpso_iter_kernel<E, UCD, false>;
+    const int blocks = grid_for(I, kern, smem, p.particles);
+    for (int64_t t = t0; t < t1; ++t) {
+        kern<<<blocks, kDpThreads, smem, s>>>(a, t);
+        const cudaError_t e = cudaGetLastError();
+        if (e != cudaSuccess) return e;
+    }
+    return cudaSuccess;
 }
 
 template <int E>
@@ -344,8 +472,8 @@ cudaError_t begin_d(Instance& I, const DpsoLaunch& p, void* ws, cudaStream_t s) 
     return p.ucd ? begin_e<E, true>(I, p, ws, s) : begin_e<E, false>(I, p, ws, s);
 }
 template <int E>
-cudaError_t iter_d(Instance& I, const DpsoLaunch& p, void* ws, int64_t t, cudaStream_t s) {
-    return p.ucd ? iter_e<E, true>(I, p, ws, t, s) : iter_e<E, false>(I, p, ws, t, s);
+cudaError_t iter_d(Instance& I, const DpsoLaunch& p, void* ws, int64_t t0, int64_t t1, cudaStream_t s) {
+    return p.ucd ? iter_e<E, true>(I, p, ws, t0, t1, s) : iter_e<E, false>(I, p, ws, t0, t1, s);
 }
 
 }  // namespace
@@ -365,14 +493,15 @@ cudaError_t dpso_begin(Instance& I, const DpsoLaunch& p, void* ws, cudaStream_t 
     }
 }
 
-cudaError_t dpso_iterate(Instance& I, const DpsoLaunch& p, void* ws, int64_t t, cudaStream_t s) {
+cudaError_t dpso_iterate(Instance& I, const DpsoLaunch& p, void* ws, int64_t t0, int64_t t1,
+                         cudaStream_t s) {
     switch (sa_e_for_n(I.n)) {
-        case 1: return iter_d<1>(I, p, ws, t, s);
-        case 2: return iter_d<2>(I, p, ws, t, s);
-        case 4: return iter_d<4>(I, p, ws, t, s);
-        case 8: return iter_d<8>(I, p, ws, t, s);
-        case 16: return iter_d<16>(I, p, ws, t, s);
-        default: return iter_d<32>(I, p, ws, t, s);
+        case 1: return iter_d<1>(I, p, ws, t0, t1, s);
+        case 2: return iter_d<2>(I, p, ws, t0, t1, s);
+        case 4: return iter_d<4>(I, p, ws, t0, t1, s);
+        case 8: return iter_d<8>(I, p, ws, t0, t1, s);
+        case 16: return iter_d<16>(I, p, ws, t0, t1, s);
+        default: return iter_d<32>(I, p, ws, t0, t1, s);
     }
 }
 

@@ -100,7 +100,9 @@ struct DpsoLaunch {
 };
 size_t dpso_workspace_bytes(const Instance& I, const DpsoLaunch& p);
 cudaError_t dpso_begin(Instance& I, const DpsoLaunch& p, void* ws, cudaStream_t s);
-cudaError_t dpso_iterate(Instance& I, const DpsoLaunch& p, void* ws, int64_t t, cudaStream_t s);
+// iterations t0..t1-1 of Alg. 2 (one kernel launch each)
+cudaError_t dpso_iterate(Instance& I, const DpsoLaunch& p, void* ws, int64_t t0, int64_t t1,
+                         cudaStream_t s);
 void dpso_gbest(const Instance& I, const DpsoLaunch& p, void* ws, int64_t t, int64_t** key,
                 int16_t** perm);
 cudaError_t dpso_end(Instance& I, const DpsoLaunch& p, void* ws, cudaStream_t s);
