@@ -110,7 +110,7 @@ def run_reference(args):
     import oracle
 
     threads = os.cpu_count() or 1
-    chains_per_thread, steps = 1, 400
+    chains_per_thread, steps = 1, 4000  # ~0.1-0.3 s of CPU work per bench step
     insts = [oracle.Problem.from_instance(gen.cdd_instance(N_JOBS, INSTANCE_SEED, h)) for h in HS]
     T0s = [oracle.t0(pr, oracle.CDD, RUN_SEED, 200) for pr in insts]
 
