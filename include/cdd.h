@@ -217,7 +217,9 @@ typedef struct {
 } dpso_params;
 CDD_API size_t dpso_workspace_size(const cdd_instance *inst, const dpso_params *params);
 /* ASYNC.  Whole run on one device (the swarm is this device's particles): lines 1-2, then
- * `iters` x lines 4-7, then the final best particle into the instance's best buffers. */
+ * `iters` x lines 4-7, then the final best particle into the instance's best buffers.
+ * CDD_EINVAL if n < 2 (F1-F3 need two positions), particles outside [1, 2^31), or the global
+ * particle ids do not fit 32 bits; iters = 0 returns the best initial particle. */
 CDD_API int dpso_run(cdd_instance *inst, const dpso_params *params, void *workspace,
              size_t workspace_bytes, void *stream);
 /* Stepping interface for a swarm spread over several GPUs.  ASYNC each.
