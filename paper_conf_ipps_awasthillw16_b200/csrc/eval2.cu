@@ -125,6 +125,17 @@ __global__ void __launch_bounds__(W * 32, 1) eval2_cdd_kernel(
     const int64_t gstep = (int64_t)gridDim.x * W;
     // this lane copies chunks cg = lane + 32 t of every sequence of a group (its stage slot
     // depends on the group only through nothing: the offsets are loop invariants)
+    // When the swizzle of a segment does not depend on the row within the group (G % 8 == 0), the
+    // stage offsets of this lane's chunks and their "before n" predicates are loop invariants.
+    constexpr bool kRowFree = G % 8 == 0;
+    uint32_t soff[X::T];
+    uint32_t pmask = 0;
+#pragma unroll
+    for (int t = 0; t < X::T; ++t) {
+        const int cg = lane + 32 * t, seg = cg / CPS, c = cg % CPS;
+        soff[t] = 16u * ((uint32_t)(seg * CPS) + ((uint32_t)c ^ X::sw(seg)));
+        if (cg < cpr) pmask |= 1u << t;
+    }
     auto issue = [&](int64_t rg, int st) {
         const uint32_t sdst = stage0 + (uint32_t)(st * X::STAGE);
 #pragma unroll
@@ -132,11 +143,17 @@ __global__ void __launch_bounds__(W * 32, 1) eval2_cdd_kernel(
             const int64_t row = rg * CPW + r;
             if (rg < ngroups && row < batch) {  // warp-uniform
                 const char* src = reinterpret_cast<const char*>(perms + row * ld) + lane * 16;
+                if constexpr (X::T > 1)  // one 64-bit address per row, not re-formed under each predicate
+                    asm("" : "+l"(src));
 #pragma unroll
                 for (int t = 0; t < X::T; ++t) {
-                    const int cg = lane + 32 * t, seg = cg / CPS, c = cg % CPS;
-                    const uint32_t slot = (uint32_t)(seg * CPS) + ((uint32_t)c ^ X::sw(r * G + seg));
-                    if (cg < cpr) cp_async16(sdst + (uint32_t)(r * X::ROWB) + 16u * slot, src + 512 * t);
+                    if constexpr (kRowFree) {
+                        if ((pmask >> t) & 1u) cp_async16(sdst + (uint32_t)(r * X::ROWB) + soff[t], src + 512 * t);
+                    } else {
+                        const int cg = lane + 32 * t, seg = cg / CPS, c = cg % CPS;
+                        const uint32_t slot = (uint32_t)(seg * CPS) + ((uint32_t)c ^ X::sw(r * G + seg));
+                        if (cg < cpr) cp_async16(sdst + (uint32_t)(r * X::ROWB) + 16u * slot, src + 512 * t);
+                    }
                 }
             }
         }
