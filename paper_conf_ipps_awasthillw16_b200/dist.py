@@ -31,6 +31,18 @@ def reduce_best(key: torch.Tensor, perm: torch.Tensor, ids_per_rank: int, group=
     return src
 
 
+def reduce_best_async(key: torch.Tensor, perm: torch.Tensor, group=None) -> None:
+    """Same result as reduce_best without a host round trip (nothing is read back): the key is
+    MIN-all-reduced, every rank but the owner (whose local key equals the minimum -- keys are
+    unique, they carry the global id) zeroes its sequence, and the sequences are SUM-all-reduced as
+    bytes, which leaves exactly the owner's.  Two collectives queued on the stream, so a loop of
+    exchanges (DPSO iterations, synchronous-SA levels) never waits on the host."""
+    local = key.clone()
+    dist.all_reduce(key, op=dist.ReduceOp.MIN, group=group)
+    perm.mul_((local == key).to(perm.dtype))
+    dist.all_reduce(perm.view(torch.uint8), op=dist.ReduceOp.SUM, group=group)
+
+
 def global_best(inst, ids_per_rank: int, group=None) -> int:
     """Reduce the instance's device-resident best (after sa_run / dpso_run) across all ranks."""
     key, perm = best_device_tensors(inst)
@@ -41,7 +53,8 @@ def dpso_run_distributed(inst, particles_per_rank: int, iters: int, problem="cdd
                          c2=0.5, seed=0, group=None, trace=False):
     """One swarm spread over all ranks (global particle ids rank*P .. rank*P+P-1).  The swarm best of
     Alg. 2 line 5 is global every iteration: after each device-local step the packed key is
-    MIN-all-reduced and the winner's sequence broadcast from its owner, then iteration t runs."""
+    MIN-all-reduced and the winner's sequence delivered to every rank (reduce_best_async: no host
+    round trip, so the iterations queue back to back), then iteration t runs."""
     from . import Dpso
 
     rank = dist.get_rank(group)
@@ -50,10 +63,10 @@ def dpso_run_distributed(inst, particles_per_rank: int, iters: int, problem="cdd
     sw.begin()
     for t in range(iters):
         key, perm = sw.gbest_tensors(t)
-        reduce_best(key, perm, particles_per_rank, group)
+        reduce_best_async(key, perm, group)
         sw.iterate(t)
     key, perm = sw.gbest_tensors(iters)
-    reduce_best(key, perm, particles_per_rank, group)
+    reduce_best_async(key, perm, group)
     sw.end()
     return sw
 
@@ -71,6 +84,6 @@ def sa_sync_run_distributed(inst, chains_per_rank: int, markov_len: int, levels:
     for j in range(levels):
         ss.level(j)
         key, perm = ss.exchange_tensors()
-        reduce_best(key, perm, chains_per_rank, group)
+        reduce_best_async(key, perm, group)
     global_best(inst, chains_per_rank, group)
     return ss

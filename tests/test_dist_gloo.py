@@ -74,3 +74,46 @@ def test_owner_rank():
 
     assert owner_rank((123 << 32) | 70000, 65536) == 1
     assert owner_rank((5 << 32) | 0, 65536) == 0
+
+
+def _worker_async(rank, world, port, q):
+    import sys
+
+    sys.path.insert(0, ROOT)
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    from paper_conf_ipps_awasthillw16_b200.dist import reduce_best, reduce_best_async
+
+    out = []
+    rng = np.random.default_rng(100 + rank)
+    for trial in range(5):
+        # penalties collide across ranks on purpose: the global id in the low word breaks ties
+        pen = int(rng.integers(0, 3))
+        gid = rank * 1000 + int(rng.integers(0, 1000))
+        perm = torch.from_numpy(rng.permutation(37).astype(np.int16))
+        k1 = torch.tensor([(pen << 32) | gid], dtype=torch.int64)
+        k2 = k1.clone()
+        p1, p2 = perm.clone(), perm.clone()
+        reduce_best(k1, p1, 1000)
+        reduce_best_async(k2, p2)
+        out.append((int(k1.item()), int(k2.item()), p1.tolist(), p2.tolist()))
+    q.put((rank, out))
+    dist.destroy_process_group()
+
+
+def test_reduce_best_async_equals_broadcast_version():
+    world = 3
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    ps = [ctx.Process(target=_worker_async, args=(r, world, port, q)) for r in range(world)]
+    [p.start() for p in ps]
+    res = dict(q.get(timeout=120) for _ in range(world))
+    [p.join(timeout=60) for p in ps]
+    assert all(p.exitcode == 0 for p in ps)
+    for trial in range(5):
+        rows = [res[r][trial] for r in range(world)]
+        k1, k2, p1, p2 = rows[0]
+        assert k1 == k2 and p1 == p2
+        assert all(r == rows[0] for r in rows)  # every rank holds the same winner
