@@ -30,7 +30,7 @@
 extern "C" {
 #endif
 
-#define CDD_ABI_VERSION 2
+#define CDD_ABI_VERSION 3
 
 #if defined(__GNUC__)
 #define CDD_API __attribute__((visibility("default")))
@@ -138,6 +138,14 @@ typedef struct {
                            /* per chain, 4 / 8 / 16 = 8 / 4 / 2 chains per warp (16-bit records: */
                            /* needs alpha, beta <= 255, else CDD_EINVAL); results do not depend  */
                            /* on it (bit-identical), only the speed does                          */
+    const int16_t *init;   /* optional device int16: Alg. 1 line 1's s0 given by the caller (P:205 */
+                           /* "the initial job sequences are copied to the GPU"): chain c (local) */
+                           /* starts from init + c * init_ld; init_ld = 0: every chain from the   */
+                           /* same sequence; init_ld >= n otherwise.  NULL: each chain's own      */
+                           /* Philox random sequence (reading R13).  Rows must be permutations of */
+                           /* 0..n-1; an id outside [0, n) raises the data-error flag (cdd_check) */
+                           /* and is replaced by 0.  Added in ABI version 3.                      */
+    int64_t init_ld;
 } sa_params;
 
 /* Bytes of device workspace sa_run needs for these parameters (caller allocates, e.g. torch). */

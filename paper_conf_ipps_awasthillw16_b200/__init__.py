@@ -43,7 +43,7 @@ class SaParams(C.Structure):
                 ("pert", C.c_int32), ("move", C.c_int), ("seed", C.c_uint64),
                 ("chain_offset", C.c_uint64), ("trace", C.c_void_p), ("chain_best", C.c_void_p),
                 ("chain_final", C.c_void_p), ("T0_out", C.c_void_p), ("T0_in", C.c_void_p),
-                ("lanes", C.c_int32)]
+                ("lanes", C.c_int32), ("init", C.c_void_p), ("init_ld", C.c_int64)]
 
 
 class SaSyncParams(C.Structure):
@@ -266,11 +266,14 @@ def sa_workspace_size(inst: Instance, **kw) -> int:
 
 def sa_run(inst: Instance, chains: int, steps: int, problem="cdd", mu=0.88, T0=0.0,
            t0_samples=5000, pert=4, move="pert_fy", seed=0, chain_offset=0, trace=False,
-           chain_best=False, chain_final=False, stream=None, workspace=None, T0_dev=None, lanes=0):
+           chain_best=False, chain_final=False, stream=None, workspace=None, T0_dev=None, lanes=0,
+           init=None):
     """Asynchronous parallel SA (Alg. 1): `chains` independent chains of `steps` iterations,
     reduced to the best (penalty, chain) into the instance's best buffers.  Returns the optional
     per-chain device tensors (and the T0 used) without synchronising.  `lanes`: threads per
-    chain (0 automatic, 32, 16, 8, 4) -- a speed knob only, results are identical."""
+    chain (0 automatic, 32, 16, 8, 4) -- a speed knob only, results are identical.  `init`:
+    optional device int16 initial sequences s0 -- [n] for every chain or [chains, ld]
+    (row c for local chain c); None: each chain's own random sequence."""
     import torch
 
     dev = torch.device("cuda", inst.device)
@@ -284,6 +287,13 @@ def sa_run(inst: Instance, chains: int, steps: int, problem="cdd", mu=0.88, T0=0
     p = _sa_params(problem, chains, steps, mu, T0, t0_samples, pert, move, seed, chain_offset,
                    res.get("trace"), res.get("chain_best"), res.get("chain_final"), res["T0"],
                    T0_dev, lanes)
+    if init is not None:
+        assert init.dtype == torch.int16 and init.is_cuda and init.stride(-1) == 1
+        assert (init.dim() == 1 and init.shape[0] >= inst.n) or (
+            init.dim() == 2 and init.shape[0] >= chains and init.shape[1] >= inst.n)
+        p.init = init.data_ptr()
+        p.init_ld = 0 if init.dim() == 1 else init.stride(0)
+        res["init"] = init  # keep alive until the (asynchronous) run is done with it
     need = int(_lib.sa_workspace_size(inst.handle, C.byref(p)))
     if need == 0:
         _check(_lib.sa_run(inst.handle, C.byref(p), None, 0, None))  # raises with the reason

@@ -344,6 +344,7 @@ static int sa_validate(const cdd_instance* I, const sa_params* p, cdd::SaLaunch*
     if (p->lanes >= 4 && p->lanes <= 16 && !I->ab16_ok)
         return fail(CDD_EINVAL, "lanes 4/8/16 need alpha, beta <= 255 (16-bit records)");
     if (p->lanes == 4 && I->n > 256) return fail(CDD_EINVAL, "lanes = 4 supports n <= 256");
+    if (p->init && p->init_ld != 0 && p->init_ld < I->n) return fail(CDD_EINVAL, "init_ld must be 0 or >= n");
     L->ucd = ucd;
     L->lanes = p->lanes;
     L->chains = p->chains;
@@ -360,6 +361,8 @@ static int sa_validate(const cdd_instance* I, const sa_params* p, cdd::SaLaunch*
     L->chain_best = p->chain_best;
     L->chain_final = p->chain_final;
     L->T0_out = p->T0_out;
+    L->init = p->init;
+    L->init_ld = p->init ? p->init_ld : 0;
     return CDD_OK;
 }
 

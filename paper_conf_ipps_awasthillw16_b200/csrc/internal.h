@@ -77,6 +77,8 @@ struct SaLaunch {
     double* T0_out;
     const double* T0_in;
     int32_t lanes;  // 0 automatic, 32 warp per chain, 4 / 8 / 16 group kernel
+    const int16_t* init = nullptr;  // caller's initial sequences (chain c: init + c * init_ld)
+    int64_t init_ld = 0;
 };
 size_t sa_workspace_bytes(const Instance& I, const SaLaunch& p);
 cudaError_t launch_t0(const Instance& I, bool ucd, uint64_t seed, int64_t samples, double* T0_dev,
