@@ -346,6 +346,7 @@ def _timed(stream, fn, reps=1):
 
 def bench_configs(lib, dev, stream):
     """Device throughput on the other BASELINE configs (one line each; CUDA-event timed)."""
+    import numpy as np
     import torch
 
     import gen
@@ -407,6 +408,28 @@ def bench_configs(lib, dev, stream):
                       "async_best_same_moves": async_best,
                       "workload": "synchronous SA, CDD n=1000 h=0.4, 65536 chains, M=50 moves x 100 "
                                   "temperature levels (mu per level)"}
+    # the headline SA from one V-shaped constructive sequence per chain instead of random ones
+    # (sa_params.init; R13): quality only, same kernel and speed
+    sys.path.insert(0, os.path.join(ROOT, "scripts"))
+    from init_quality import v_shaped_candidates
+
+    bk_path = os.path.join(ROOT, "tests", "golden", "best_known_n1000.json")
+    bk = json.load(open(bk_path))["best_known"] if os.path.exists(bk_path) else {}
+    vq = {}
+    for h in HS:
+        g = gen.cdd_instance(N_JOBS, INSTANCE_SEED, h)
+        ins = lib.Instance.from_gen(g, device=dev.index)
+        cands = torch.from_numpy(v_shaped_candidates(g, np.linspace(0.2, 1.0, 33))).to(dev)
+        s0 = cands[int(torch.argmin(lib.cdd_eval_batch(ins, cands)).item())].contiguous()
+        lib.sa_run(ins, CHAINS, SA_STEPS, seed=RUN_SEED, t0_samples=T0_SAMPLES, init=s0)
+        pen, _, _ = lib.best_get(ins)
+        key = f"{h:.1f}"
+        vq[key] = {"best": pen}
+        if key in bk:
+            vq[key]["gap_pct"] = 100.0 * (pen - bk[key]) / bk[key]
+    out["sa_from_v_shaped_start"] = {
+        "quality": vq, "workload": "config 5 SA (65536 chains x 5000 steps) with every chain "
+                                   "starting from one V-shaped constructive sequence (scripts/init_quality.py)"}
     return out
 
 
