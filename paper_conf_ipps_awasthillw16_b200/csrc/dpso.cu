@@ -107,9 +107,10 @@ __global__ void __launch_bounds__(kDpThreads) dpso_init_kernel(DpArgs a) {
     for (int64_t i = (int64_t)blockIdx.x * kDpWarps + wib; i < a.particles; i += total) {
         const uint64_t gid = a.offset + (uint64_t)i;
         chain_fy_init<E, UCD>(ch, a.n, a.seed, kTagDpsoInit, gid, lane);
-        // positions past n carry the sentinel id NP - 1 (>= n: a zero record in the iteration
-        // kernel's table); the crossovers never move them
-        for (int k = a.n + lane; k < C::NP; k += 32) ch.id()[k] = (uint16_t)(C::NP - 1);
+        // position k >= n carries the sentinel id k (>= n: a zero record in the iteration kernel's
+        // table; distinct, so the position-of-job writes of the pads never collide); the
+        // crossovers never move them
+        for (int k = a.n + lane; k < C::NP; k += 32) ch.id()[k] = (uint16_t)k;
         __syncwarp();
         chain_build<E, UCD>(ch, a.T, a.n, lane);
         const int32_t z = chain_eval<E, UCD>(ch, lane, a.n, a.d);
@@ -295,7 +296,7 @@ __global__ void __launch_bounds__(kDpThreads) dpso_iter_kernel(DpArgs a, int64_t
                 const uint4 x = __ldg(reinterpret_cast<const uint4*>(gp + o));
                 *reinterpret_cast<uint4*>(ids + o) = x;
                 const uint32_t w[4] = {x.x, x.y, x.z, x.w};
-#pragma unroll  // (positions past n hold the sentinel NP - 1, whose entry is never read)
+#pragma unroll  // (position k >= n holds the sentinel id k: distinct entries, never read)
                 for (int j = 0; j < 8; ++j)
                     inv[(j & 1) ? (w[j >> 1] >> 16) : (w[j >> 1] & 0xffffu)] = (uint16_t)(o + j);
             }

@@ -1,0 +1,31 @@
+"""Small runs of every kernel family for compute-sanitizer (memcheck / racecheck / synccheck):
+python scripts/sanitize.py  (under `compute-sanitizer --tool X python scripts/sanitize.py`)."""
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+
+import torch  # noqa: E402
+
+import gen  # noqa: E402
+import paper_conf_ipps_awasthillw16_b200 as cdd  # noqa: E402
+
+for n in (7, 50, 100, 200, 500, 777, 1000):
+    ins = cdd.Instance.from_gen(gen.cdd_instance(n, 1, 0.4))
+    perms = gen.random_perms_device(700, n, 3, ld=(n + 7) // 8 * 8)
+    cdd.cdd_eval_batch(ins, perms)
+    cdd.cdd_schedule_batch(ins, perms[:50])
+    cdd.sa_run(ins, 300, 20, seed=1, t0_samples=100)
+    cdd.sa_run(ins, 40, 20, seed=1, t0_samples=100, lanes=32, init=perms[0])
+    if n >= 2:
+        cdd.dpso_run(ins, 64, 5, seed=2)
+    cdd.SaSync(ins, 64, 5, 3, seed=3, t0_samples=100).run()
+    cdd.cdd_check(ins)
+    u = cdd.Instance.from_gen(gen.ucddcp_instance(n, 1))
+    cdd.ucddcp_eval_batch(u, perms)
+    cdd.sa_run(u, 300, 20, problem="ucddcp", seed=1, t0_samples=100)
+    if n >= 2:
+        cdd.dpso_run(u, 64, 5, problem="ucddcp", seed=2)
+    cdd.cdd_check(u)
+torch.cuda.synchronize()
+print("sanitize run ok")
