@@ -31,7 +31,8 @@ HS = (0.2, 0.4, 0.6, 0.8)
 INSTANCE_SEED = 1
 RUN_SEED = 0x5EED0005
 METRIC = "sequence evals/s at n=1000 on 1/8 B200; SA % gap vs best-known"
-WORKLOAD = "config5: CDD n=1000, h in {0.2,0.4,0.6,0.8} (instance seed 1), 65536 SA chains/GPU x 5000 steps, T0 from 5000 samples"
+WORKLOAD = ("config5: CDD n=1000, h in {{0.2,0.4,0.6,0.8}} (instance seed 1), {chains} SA chains/GPU x "
+            "{steps} steps, T0 from 5000 samples")
 INT_OPS_PER_ELEM = 6  # 3 prefix adds + subtract + select + multiply-add per job
 
 
@@ -137,7 +138,7 @@ def run_reference(args):
             "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": 1000 * sum(dts) / args.steps, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "int32", "data": "synthetic",
-            "config": {"workload": WORKLOAD, "sample": sample},
+            "config": {"workload": WORKLOAD.format(chains=CHAINS, steps=SA_STEPS), "sample": sample},
             "cpu_baseline": {"value": value, "unit": "evals/s", "cores": threads, "kind": "oracle",
                              "sample": sample},
             "e2e": {"value": value, "unit": "evals/s", "h2d_bytes_per_step": 0,
@@ -202,9 +203,16 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    # CDD_BENCH_DEVICES=k maps local ranks onto k GPUs (test hook: several ranks on one GPU need
+    # CDD_BENCH_BACKEND=gloo, NCCL refuses duplicate devices); default one GPU per rank, NCCL
+    local = local % int(os.environ.get("CDD_BENCH_DEVICES", str(max(1, torch.cuda.device_count()))))
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        backend = os.environ.get("CDD_BENCH_BACKEND", "nccl")
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
     dev = torch.device("cuda", local)
     stream = torch.cuda.current_stream(dev)
 
@@ -315,7 +323,8 @@ def main():
                 "steps": args.steps, "warmup": args.warmup, "ms_per_step": step_ms,
                 "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
                 "dtype": "int32", "data": "synthetic",
-                "config": {"workload": WORKLOAD, "n": N_JOBS, "chains_per_gpu": chains,
+                "config": {"workload": WORKLOAD.format(chains=chains, steps=steps), "n": N_JOBS,
+                           "chains_per_gpu": chains,
                            "sa_steps": steps, "t0_samples": T0_SAMPLES, "instances": len(insts),
                            "parallelism": f"dp{world} (independent chains, NCCL min-allreduce)",
                            "l2": "state is on-chip; L2 flushed (256 MiB write) before every instance"},
