@@ -1,8 +1,9 @@
 // schedule.cu -- the optimal schedule of a sequence: what the O(n) timing
 // routine finds, not just its cost.
 //
-// One warp per sequence, lane L owns positions [L*E, L*E+E) (E = ceil(n/32)); the job data is read
-// through the id tables (global, L1-resident).  Same quantities as the evaluators:
+// One warp per sequence, lane L owns positions [L*E, L*E+E) (E = pow2 >= ceil(n/32)); the ids
+// are staged in shared memory by coalesced loads, the job data is read from tables staged per
+// CTA, and the rows of C (and X) are assembled in shared memory and written out coalesced.  Same quantities as the evaluators:
 //   S_k = sum_{j<k} (alpha_j + beta_j), k0 = max{k : S_k <= Btot}, C_k = sum_{j<=k} p_j;
 //   CDD:    D = min(C_{k0}, d); the first job starts at s = d - D >= 0 (job k0 completes at d
 //           when C_{k0} <= d, else the schedule starts at time 0), C_k <- s + C_k;
@@ -52,27 +53,91 @@ __device__ __forceinline__ int64_t warp_sum64(int64_t v) {
     return v;
 }
 
-template <bool UCD>
-__global__ void __launch_bounds__(128) schedule_kernel(SchedArgs a) {
-    const int lane = threadIdx.x & 31;
-    const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
-    const int n = a.n, E = (n + 31) / 32, k_lo = lane * E, k_hi = min(n, k_lo + E);
+// Shared-memory layout (dynamic): the instance tables by job id (ab u32, p u8 [, M u8, X u8,
+// gamma u16], each array padded to 16 bytes), then per warp: the sequence's ids in lane segments
+// of E positions (E = pow2 >= ceil(n/32), segments padded by 16 bytes), and the output staging
+// C (int64) [and X (int32)] in lane segments padded by one element, so that the lane-contiguous
+// compute writes and the coalesced copy-out reads are both (nearly) conflict free.
+struct SchedLayout {
+    int n, E, lE;
+    uint32_t tab_bytes, ids_off, c_off, x_off, warp_bytes, total;
+};
+__host__ __device__ inline uint32_t al16(uint32_t x) { return (x + 15u) & ~15u; }
+__host__ __device__ inline SchedLayout sched_layout(int n, bool ucd, int warps) {
+    SchedLayout L{};
+    L.n = n;
+    L.lE = 0;
+    while ((32 << L.lE) < n) ++L.lE;
+    L.E = 1 << L.lE;
+    const uint32_t N = (uint32_t)n;
+    L.tab_bytes = al16(4 * (N + 1)) + al16(N + 1) + (ucd ? al16(N + 1) + al16(N + 1) + al16(2 * (N + 1)) : 0u);
+    L.ids_off = 0;
+    L.c_off = al16(32u * (2u * L.E + 16u));
+    L.x_off = L.c_off + al16(32u * 8u * (L.E + 1u));
+    L.warp_bytes = L.x_off + (ucd ? al16(32u * 4u * (L.E + 1u)) : 0u);
+    L.total = L.tab_bytes + (uint32_t)warps * L.warp_bytes;
+    return L;
+}
+constexpr int kSchedWarps = 4;
+
+template <bool UCD, int E>
+__global__ void __launch_bounds__(kSchedWarps * 32) schedule_kernel(SchedArgs a) {
+    extern __shared__ __align__(16) uint8_t smem[];
+    const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+    const int n = a.n;
+    const SchedLayout Ly = sched_layout(n, UCD, kSchedWarps);  // (its E equals the template's)
+    constexpr int lE = E == 1 ? 0 : E == 2 ? 1 : E == 4 ? 2 : E == 8 ? 3 : E == 16 ? 4 : 5;
+    const uint32_t N = (uint32_t)n;
+    // CTA tables
+    // (entry n is the zero record of the sentinel id that pads the lane segments past n: padded
+    // slots add nothing to any sum, and where they pass the S <= Btot test -- only if every alpha
+    // is 0 -- they repeat C_{n-1}, so no slot needs an index test)
+    uint32_t* t_ab = reinterpret_cast<uint32_t*>(smem);
+    uint8_t* t_p = smem + al16(4 * (N + 1));
+    uint8_t* t_m = t_p + al16(N + 1);
+    uint8_t* t_x = t_m + al16(N + 1);
+    uint16_t* t_g = reinterpret_cast<uint16_t*>(t_x + al16(N + 1));
+    for (int j = threadIdx.x; j <= n; j += blockDim.x) {
+        const bool v = j < n;
+        t_ab[j] = v ? __ldg(a.ab + j) : 0u;
+        t_p[j] = v ? __ldg(a.p + j) : (uint8_t)0;
+        if constexpr (UCD) {
+            t_m[j] = v ? __ldg(a.m + j) : (uint8_t)0;
+            t_x[j] = v ? __ldg(a.x + j) : (uint8_t)0;
+            t_g[j] = v ? __ldg(a.g + j) : (uint16_t)0;
+        }
+    }
+    uint8_t* wbase = smem + Ly.tab_bytes + (size_t)wib * Ly.warp_bytes;
+    uint16_t* ids_s = reinterpret_cast<uint16_t*>(wbase + Ly.ids_off);
+    int64_t* C_s = reinterpret_cast<int64_t*>(wbase + Ly.c_off);
+    int32_t* X_s = reinterpret_cast<int32_t*>(wbase + Ly.x_off);
+    const int IS = E + 8, CS = E + 1;  // segment strides (elements)
+    const int k_lo = lane * E;
+    // loops below run over all E slots of the lane's segment (unrolled); slots past n hold id n
+    for (int k = n + lane; k < 32 * E; k += 32) ids_s[(k >> lE) * IS + (k & (E - 1))] = (uint16_t)n;
+    __syncthreads();
+    const uint16_t* myids = ids_s + lane * IS;
+    int64_t* myC = C_s + lane * CS;
+    int32_t* myX = X_s + lane * CS;
+    const int64_t warps = (int64_t)gridDim.x * kSchedWarps;
     bool bad = false;
-    for (int64_t row = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); row < a.batch;
-         row += warps) {
+    for (int64_t row = (int64_t)blockIdx.x * kSchedWarps + wib; row < a.batch; row += warps) {
         const int16_t* rp = a.perms + row * a.ld;
-        auto job = [&](int k) -> int {
+        // ids, coalesced, validated (an id outside [0, n) raises the flag and reads job 0)
+        for (int k = lane; k < n; k += 32) {
             const int id = rp[k];
             const bool ok = id >= 0 && id < n;
             bad |= !ok;
-            return ok ? id : 0;
-        };
+            ids_s[(k >> lE) * IS + (k & (E - 1))] = (uint16_t)(ok ? id : 0);
+        }
+        __syncwarp();
         // lane totals, then exclusive bases
         int32_t tP = 0, tA = 0, tB = 0;
-        for (int k = k_lo; k < k_hi; ++k) {
-            const int j = job(k);
-            const uint32_t r = __ldg(a.ab + j);
-            tP += __ldg(a.p + j);
+        #pragma unroll
+        for (int i = 0; i < E; ++i) {
+            const int j = myids[i];
+            const uint32_t r = t_ab[j];
+            tP += t_p[j];
             tA += (int32_t)(r & 0xffffu);
             tB += (int32_t)(r >> 16);
         }
@@ -84,12 +149,13 @@ __global__ void __launch_bounds__(128) schedule_kernel(SchedArgs a) {
         int32_t Ck0 = 0;
         {
             int32_t c = Pb, s = Ab + Bb;
-            for (int k = k_lo; k < k_hi; ++k) {
-                const int j = job(k);
-                const uint32_t r = __ldg(a.ab + j);
-                c += __ldg(a.p + j);
+            #pragma unroll
+        for (int i = 0; i < E; ++i) {
+                const int j = myids[i];
+                const uint32_t r = t_ab[j];
+                c += t_p[j];
                 if (s <= Btot) {
-                    k0 = k;
+                    k0 = k_lo + i;
                     Ck0 = c;
                 }
                 s += (int32_t)(r & 0xffffu) + (int32_t)(r >> 16);
@@ -99,38 +165,34 @@ __global__ void __launch_bounds__(128) schedule_kernel(SchedArgs a) {
         const int owner = 31 - __clz(has);  // lane 0 always has k = 0 (S_0 = 0 <= Btot)
         k0 = __shfl_sync(kFull, k0, owner);
         Ck0 = __shfl_sync(kFull, Ck0, owner);
-        int64_t* Crow = a.C + row * (int64_t)n;
         int64_t pen = 0;
+        int64_t st = 0;
         if constexpr (!UCD) {
             const int64_t D = min((int64_t)Ck0, a.d);
-            const int64_t s0 = a.d - D;  // start of the first job
-            int64_t c = s0 + Pb;
-            for (int k = k_lo; k < k_hi; ++k) {
-                const int j = job(k);
-                const uint32_t r = __ldg(a.ab + j);
-                c += __ldg(a.p + j);
-                Crow[k] = c;
+            st = a.d - D;  // start of the first job
+            int64_t c = st + Pb;
+            #pragma unroll
+        for (int i = 0; i < E; ++i) {
+                const int j = myids[i];
+                const uint32_t r = t_ab[j];
+                c += t_p[j];
+                myC[i] = c;
                 pen += (int64_t)(r & 0xffffu) * max((int64_t)0, a.d - c) +
                        (int64_t)(r >> 16) * max((int64_t)0, c - a.d);
             }
-            pen = warp_sum64(pen);
-            if (lane == 0) {
-                a.start[row] = s0;
-                a.pen[row] = pen;
-            }
         } else {
-            int32_t* Xrow = a.X + row * (int64_t)n;
             // compression decisions and the lane totals of p'
             int32_t tQ = 0;
             {
                 int32_t A = Ab, B = Bb;  // exclusive prefixes
-                for (int k = k_lo; k < k_hi; ++k) {
-                    const int j = job(k);
-                    const uint32_t r = __ldg(a.ab + j);
-                    const int32_t w = k <= k0 ? A : Btot - B;
-                    const int32_t xk = w > (int32_t)__ldg(a.g + j) ? (int32_t)__ldg(a.x + j) : 0;
-                    Xrow[k] = xk;
-                    tQ += (int32_t)__ldg(a.m + j) + (int32_t)__ldg(a.x + j) - xk;
+                #pragma unroll
+        for (int i = 0; i < E; ++i) {
+                    const int j = myids[i];
+                    const uint32_t r = t_ab[j];
+                    const int32_t w = k_lo + i <= k0 ? A : Btot - B;
+                    const int32_t xk = w > (int32_t)t_g[j] ? (int32_t)t_x[j] : 0;
+                    myX[i] = xk;
+                    tQ += (int32_t)t_m[j] + (int32_t)t_x[j] - xk;
                     A += (int32_t)(r & 0xffffu);
                     B += (int32_t)(r >> 16);
                 }
@@ -140,31 +202,42 @@ __global__ void __launch_bounds__(128) schedule_kernel(SchedArgs a) {
             int32_t Qk0 = 0;
             {
                 int32_t q = Qb;
-                for (int k = k_lo; k < k_hi; ++k) {
-                    const int j = job(k);
-                    q += (int32_t)__ldg(a.m + j) + (int32_t)__ldg(a.x + j) - Xrow[k];
-                    if (k == k0) Qk0 = q;
+                #pragma unroll
+        for (int i = 0; i < E; ++i) {
+                    const int j = myids[i];
+                    q += (int32_t)t_m[j] + (int32_t)t_x[j] - myX[i];
+                    if (k_lo + i == k0) Qk0 = q;
                 }
             }
             Qk0 = __shfl_sync(kFull, Qk0, owner);
+            st = a.d - Qk0;
             int32_t q = Qb;
-            for (int k = k_lo; k < k_hi; ++k) {
-                const int j = job(k);
-                const uint32_t r = __ldg(a.ab + j);
-                const int32_t xk = Xrow[k];
-                q += (int32_t)__ldg(a.m + j) + (int32_t)__ldg(a.x + j) - xk;
+            #pragma unroll
+        for (int i = 0; i < E; ++i) {
+                const int j = myids[i];
+                const uint32_t r = t_ab[j];
+                const int32_t xk = myX[i];
+                q += (int32_t)t_m[j] + (int32_t)t_x[j] - xk;
                 const int64_t c = a.d - (int64_t)(Qk0 - q);
-                Crow[k] = c;
+                myC[i] = c;
                 pen += (int64_t)(r & 0xffffu) * max((int64_t)0, a.d - c) +
-                       (int64_t)(r >> 16) * max((int64_t)0, c - a.d) +
-                       (int64_t)__ldg(a.g + j) * xk;
-            }
-            pen = warp_sum64(pen);
-            if (lane == 0) {
-                a.start[row] = a.d - Qk0;
-                a.pen[row] = pen;
+                       (int64_t)(r >> 16) * max((int64_t)0, c - a.d) + (int64_t)t_g[j] * xk;
             }
         }
+        pen = warp_sum64(pen);
+        if (lane == 0) {
+            a.start[row] = st;
+            a.pen[row] = pen;
+        }
+        __syncwarp();
+        // coalesced copy-out of the staged rows
+        int64_t* Crow = a.C + row * (int64_t)n;
+        for (int k = lane; k < n; k += 32) Crow[k] = C_s[(k >> lE) * CS + (k & (E - 1))];
+        if constexpr (UCD) {
+            int32_t* Xrow = a.X + row * (int64_t)n;
+            for (int k = lane; k < n; k += 32) Xrow[k] = X_s[(k >> lE) * CS + (k & (E - 1))];
+        }
+        __syncwarp();
     }
     if (bad) atomicOr(a.err, 1);
 }
@@ -177,12 +250,27 @@ cudaError_t launch_schedule(const Instance& I, bool ucd, const int16_t* perms, i
     if (batch == 0) return cudaSuccess;
     SchedArgs a{I.tab_ab, I.tab_p, I.tab_m, I.tab_x, I.tab_g, I.n, I.d, perms, ld, batch,
                 C, start, pen, X, I.err};
-    int sms = 148;
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, I.device);
-    const int64_t want = (batch + 3) / 4;
-    const int blocks = (int)(want < (int64_t)sms * 16 ? want : (int64_t)sms * 16);
-    if (ucd) schedule_kernel<true><<<blocks, 128, 0, s>>>(a);
-    else schedule_kernel<false><<<blocks, 128, 0, s>>>(a);
+    const SchedLayout Ly = sched_layout(I.n, ucd, kSchedWarps);
+    void (*kern)(SchedArgs) = nullptr;
+    switch (Ly.E) {
+        case 1: kern = ucd ? schedule_kernel<true, 1> : schedule_kernel<false, 1>; break;
+        case 2: kern = ucd ? schedule_kernel<true, 2> : schedule_kernel<false, 2>; break;
+        case 4: kern = ucd ? schedule_kernel<true, 4> : schedule_kernel<false, 4>; break;
+        case 8: kern = ucd ? schedule_kernel<true, 8> : schedule_kernel<false, 8>; break;
+        case 16: kern = ucd ? schedule_kernel<true, 16> : schedule_kernel<false, 16>; break;
+        default: kern = ucd ? schedule_kernel<true, 32> : schedule_kernel<false, 32>; break;
+    }
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)Ly.total);
+    if (e != cudaSuccess) return e;
+    int sms = 148, occ = 1;
+    e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, I.device);
+    if (e != cudaSuccess) return e;
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kSchedWarps * 32, Ly.total);
+    if (e != cudaSuccess) return e;
+    const int64_t want = (batch + kSchedWarps - 1) / kSchedWarps;
+    const int64_t cap = (int64_t)sms * (occ < 1 ? 1 : occ);
+    const int blocks = (int)(want < cap ? want : cap);
+    kern<<<blocks, kSchedWarps * 32, Ly.total, s>>>(a);
     return cudaGetLastError();
 }
 

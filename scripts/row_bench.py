@@ -1,0 +1,111 @@
+"""One measurement per SURVEY §8 row that has a kernel of its own, each against the roofline that
+bounds it (DESIGN.md §7 / §8): prints one JSON line per row.
+
+  A7  cdd_eval_batch / ucddcp_eval_batch, n=1000: HBM (2n + 8 bytes per sequence)
+  A8  T0 rule (5000 samples), n=1000: issue (6n integer ops per sampled evaluation)
+  A9-A11 asynchronous SA, n=1000: issue (6n per evaluation; UCDDCP 9n)
+  A13-A14 DPSO, n=500: issue (6n per particle evaluation)
+  F1  cdd_schedule_batch, n=1000: HBM (2n read + 8n written + 16 bytes per sequence)
+  F2  synchronous SA, n=1000: issue (6n per evaluation)
+
+Peaks: MEASURED_PEAKS.json (HBM GB/s, SM max clock); integer issue peak = 128 lane-ops/clk/SM x SMs
+x max clock.  Inputs larger than L2 for the HBM rows (two alternating pools).
+python scripts/row_bench.py"""
+import json
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import torch  # noqa: E402
+
+import gen  # noqa: E402
+import paper_conf_ipps_awasthillw16_b200 as cdd  # noqa: E402
+
+
+def timed(fn, reps=5):
+    fn()
+    torch.cuda.synchronize()
+    ts = []
+    for r in range(reps):
+        s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        s.record()
+        fn(r)
+        e.record()
+        torch.cuda.synchronize()
+        ts.append(s.elapsed_time(e) / 1000.0)
+    return sorted(ts)[len(ts) // 2]
+
+
+def main():
+    peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json"))) if os.path.exists(
+        os.path.join(ROOT, "MEASURED_PEAKS.json")) else {}
+    hbm = float(peaks.get("hbm_gbs", 6454.0))
+    sm_mhz = float(peaks.get("sm_max_mhz", 1965.0))
+    nsm = torch.cuda.get_device_properties(0).multi_processor_count
+    alu = 128 * nsm * sm_mhz * 1e6 / 1e12  # T int-op/s
+
+    def out(row, what, value, unit, achieved, peak, punit, note=""):
+        print(json.dumps({"row": row, "what": what, "value": value, "unit": unit,
+                          "roofline": {"achieved": achieved, "peak": peak, "unit": punit,
+                                       "frac": achieved / peak}, "note": note}), flush=True)
+
+    n = 1000
+    rows = 1 << 20
+    pools = [gen.random_perms_device(rows, n, seed=s, ld=n) for s in (1, 2)]
+    o = torch.empty(rows, dtype=torch.int64, device="cuda")
+    ic = cdd.Instance.from_gen(gen.cdd_instance(n, 1, 0.4))
+    iu = cdd.Instance.from_gen(gen.ucddcp_instance(n, 1))
+    for name, ins, fn in (("cdd_eval_batch", ic, cdd.cdd_eval_batch), ("ucddcp_eval_batch", iu, cdd.ucddcp_eval_batch)):
+        dt = timed(lambda r=0: fn(ins, pools[r & 1], o), reps=9)
+        gbs = rows * (2 * n + 8) / dt / 1e9
+        out("A7" if name.startswith("cdd") else "A6/A7", f"{name} n={n}, 2^20 sequences", rows / dt,
+            "evals/s", gbs, hbm, "GB/s")
+    cdd.cdd_check(ic)
+    cdd.cdd_check(iu)
+
+    # F1 schedules: C int64 [B, n] written, sequences read
+    B = 1 << 17
+    sp = pools[0][:B]
+    dt = timed(lambda r=0: cdd.cdd_schedule_batch(ic, sp), reps=5)
+    out("F1", f"cdd_schedule_batch n={n}, 2^17 sequences", B / dt, "schedules/s",
+        B * (2 * n + 8 * n + 16) / dt / 1e9, hbm, "GB/s", "C int64 [B, n] written + start + penalty")
+
+    # A8 T0
+    T0 = 5000
+    dt = timed(lambda r=0: cdd.sa_t0(ic, seed=r, samples=T0), reps=9)
+    out("A8", f"T0 rule, {T0} samples, n={n}", T0 / dt, "samples/s", 6 * n * T0 / dt / 1e12, alu,
+        "Tint-op/s", "one launch pair: small grid (5000 warps), latency-bound")
+
+    # A9-A11 SA (CDD and UCDDCP)
+    for prob, ins, ops in (("cdd", ic, 6), ("ucddcp", iu, 9)):
+        C, S = 65536, 1000
+        t0 = cdd.sa_t0(ins, problem=prob, seed=1, samples=T0)
+        ws = cdd.sa_run(ins, C, S, problem=prob, seed=1, T0_dev=t0)["workspace"]
+        dt = timed(lambda r=0: cdd.sa_run(ins, C, S, problem=prob, seed=1, T0_dev=t0, workspace=ws), reps=3)
+        ev = C * (S + 1)
+        out("A9-A11", f"SA {prob} n={n}, {C} chains x {S} steps", ev / dt, "evals/s",
+            ops * n * ev / dt / 1e12, alu, "Tint-op/s", f"{ops}n algorithmic int ops per evaluation")
+
+    # F2 synchronous SA
+    C, M, L = 65536, 50, 20
+    ss = cdd.SaSync(ic, C, M, L, seed=3, t0_samples=T0, level_min=False)
+    dt = timed(lambda r=0: ss.run(), reps=3)
+    ev = C * M * L
+    out("F2", f"synchronous SA n={n}, {C} chains, M={M} x {L} levels", ev / dt, "evals/s",
+        6 * n * ev / dt / 1e12, alu, "Tint-op/s")
+
+    # A13-A14 DPSO
+    n2 = 500
+    i5 = cdd.Instance.from_gen(gen.cdd_instance(n2, 1, 0.6))
+    P, it = 8192, 200
+    sw = cdd.Dpso(i5, P, it, seed=4)
+    dt = timed(lambda r=0: sw.run(), reps=3)
+    ev = P * (it + 1)
+    out("A13-A14", f"DPSO n={n2}, {P} particles x {it} iterations", ev / dt, "particle-evals/s",
+        6 * n2 * ev / dt / 1e12, alu, "Tint-op/s", "per iteration: F1-F3 + evaluation + swarm best")
+
+
+if __name__ == "__main__":
+    main()
