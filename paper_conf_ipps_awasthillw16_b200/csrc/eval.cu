@@ -416,8 +416,9 @@ cudaError_t launch_eval_batch(const Instance& I, bool ucd, const int16_t* perms,
                               int64_t batch, int64_t* out, cudaStream_t s) {
     if (batch <= 0) return cudaSuccess;
 #ifndef CDD_EVAL_V1
-    if (!ucd) {
-        const cudaError_t e = launch_eval2_cdd(I, perms, ld, batch, out, s);
+    {
+        const cudaError_t e = ucd ? launch_eval2_ucddcp(I, perms, ld, batch, out, s)
+                                  : launch_eval2_cdd(I, perms, ld, batch, out, s);
         if (e != cudaErrorNotSupported) return e;
     }
 #endif

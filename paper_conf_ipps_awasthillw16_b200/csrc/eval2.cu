@@ -59,6 +59,16 @@ __device__ __forceinline__ uint32_t ldtab(uint32_t addr) {
     return v;
 }
 
+template <uint32_t TOFF>
+__device__ __forceinline__ uint2 ldtab64(uint32_t addr) {
+    uint2 v;
+    if constexpr (TOFF == 0)
+        asm volatile("ld.shared.v2.u32 {%0,%1}, [%2];" : "=r"(v.x), "=r"(v.y) : "r"(addr));
+    else
+        asm volatile("ld.shared.v2.u32 {%0,%1}, [%2+%3];" : "=r"(v.x), "=r"(v.y) : "r"(addr), "n"(TOFF));
+    return v;
+}
+
 __device__ __forceinline__ uint4 lds128(uint32_t addr) {
     uint4 v;
     asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(addr));
@@ -90,10 +100,38 @@ struct E2 {
     static __device__ __forceinline__ uint32_t sw(int S) { return (uint32_t)((S * CPS / 8) % CPS); }
 };
 
+// Job ids of positions e0 .. e0+SPR-1 of the staged lane segment at bseg (swizzle bsw), as
+// 16-bit pairs.
+template <int G, int E, int SPR>
+__device__ __forceinline__ void e2_row_ids(uint32_t bseg, uint32_t bsw, int e0, uint32_t (&idw)[(SPR + 1) / 2]) {
+    if constexpr (SPR >= 8) {
+#pragma unroll
+        for (int v = 0; v < SPR / 8; ++v) {
+            const uint4 q = lds128(bseg + ((((uint32_t)(e0 / 8 + v)) ^ bsw) << 4));
+            idw[4 * v] = q.x; idw[4 * v + 1] = q.y; idw[4 * v + 2] = q.z; idw[4 * v + 3] = q.w;
+        }
+    } else {
+        const uint32_t a = bseg + ((((uint32_t)(e0 / 8)) ^ bsw) << 4) + (uint32_t)((e0 % 8) * 2);
+        if constexpr (SPR == 4) {
+            uint32_t x0, x1;
+            asm volatile("ld.shared.v2.u32 {%0,%1}, [%2];" : "=r"(x0), "=r"(x1) : "r"(a));
+            idw[0] = x0; idw[1] = x1;
+        } else if constexpr (SPR == 2) {
+            idw[0] = lds32(a);
+        } else {
+            uint32_t x;
+            asm volatile("ld.shared.u16 %0, [%1];" : "=r"(x) : "r"(a));
+            idw[0] = x;
+        }
+    }
+}
+
 // One group of 32/G sequences per warp and stage.
-template <int G, int E, int W, uint32_t TOFF, bool TAIL>
-__global__ void __launch_bounds__(W * 32, 1) eval2_cdd_kernel(
-    const uint16_t* __restrict__ tab_ab16, const uint8_t* __restrict__ tab_p, int n, int npow2,
+template <int G, int E, int W, uint32_t TOFF, bool TAIL, bool UCD>
+__global__ void __launch_bounds__(W * 32, 1) eval2_kernel(
+    const uint16_t* __restrict__ tab_ab16, const uint8_t* __restrict__ tab_p,
+    const uint8_t* __restrict__ tab_m, const uint8_t* __restrict__ tab_x,
+    const uint16_t* __restrict__ tab_g, int n, int npow2,
     int kc_log2, int32_t d, const int16_t* __restrict__ perms, int64_t ld, int64_t batch,
     int64_t* __restrict__ out, int* __restrict__ err) {
     using X = E2<G, E>;
@@ -103,21 +141,33 @@ __global__ void __launch_bounds__(W * 32, 1) eval2_cdd_kernel(
     const int grp = lane / G, l = lane % G, gbase = grp * G;
     const int KC = 1 << kc_log2;
     const uint32_t sbase = (uint32_t)__cvta_generic_to_shared(smem);
-    const uint32_t tbytes = (uint32_t)npow2 * 4u * (uint32_t)KC;
+    constexpr uint32_t RB = UCD ? 8u : 4u;  // bytes per table entry
+    const uint32_t tbytes = (uint32_t)npow2 * RB * (uint32_t)KC;
     const E2Layout Ly = TOFF ? E2Layout{0u, 0u, tbytes + (uint32_t)W * 2u * X::STAGE}
                              : e2_layout(sbase, tbytes, 2u * X::STAGE, W);
     const uint32_t tab = TOFF ? 0u : sbase + Ly.tab_off;
     const uint32_t stage0 = sbase + ((uint32_t)warp < Ly.nb ? (uint32_t)warp * 2u * X::STAGE
                                                               : Ly.tab_off + tbytes + ((uint32_t)warp - Ly.nb) * 2u * X::STAGE);
-    uint32_t* s_tab = reinterpret_cast<uint32_t*>(smem + Ly.tab_off);
-    for (int i = threadIdx.x; i < npow2 * KC; i += blockDim.x) {
-        const int id = i >> kc_log2;
-        s_tab[i] = id < n ? (uint32_t)__ldg(tab_ab16 + id) | ((uint32_t)__ldg(tab_p + id) << 16) : 0u;
+    if constexpr (UCD) {
+        // alpha | beta << 8 | gamma << 16,  M | X << 8
+        uint2* s_tab = reinterpret_cast<uint2*>(smem + Ly.tab_off);
+        for (int i = threadIdx.x; i < npow2 * KC; i += blockDim.x) {
+            const int id = i >> kc_log2;
+            s_tab[i] = id < n ? make_uint2((uint32_t)__ldg(tab_ab16 + id) | ((uint32_t)__ldg(tab_g + id) << 16),
+                                           (uint32_t)__ldg(tab_m + id) | ((uint32_t)__ldg(tab_x + id) << 8))
+                              : make_uint2(0u, 0u);
+        }
+    } else {
+        uint32_t* s_tab = reinterpret_cast<uint32_t*>(smem + Ly.tab_off);
+        for (int i = threadIdx.x; i < npow2 * KC; i += blockDim.x) {
+            const int id = i >> kc_log2;
+            s_tab[i] = id < n ? (uint32_t)__ldg(tab_ab16 + id) | ((uint32_t)__ldg(tab_p + id) << 16) : 0u;
+        }
     }
     __syncthreads();
-    const int SH = 2 + kc_log2;  // log2(4 bytes * KC copies)
-    const uint32_t amask = tbytes - 4u * (uint32_t)KC;
-    const uint32_t tabc = tab | (uint32_t)((lane & (KC - 1)) * 4);
+    const int SH = (UCD ? 3 : 2) + kc_log2;  // log2(RB bytes * KC copies)
+    const uint32_t amask = tbytes - RB * (uint32_t)KC;
+    const uint32_t tabc = tab | (uint32_t)(lane & (KC - 1)) * RB;
 
     const int cpr = (n + 7) / 8;  // 16-byte chunks of real ids per sequence (ld % 8 == 0)
     const uint32_t S = (uint32_t)npow2 - 1u;  // sentinel id: >= n, zero record
@@ -194,9 +244,6 @@ __global__ void __launch_bounds__(W * 32, 1) eval2_cdd_kernel(
         const uint32_t srow = stage0 + (uint32_t)(st * X::STAGE) + (uint32_t)(grp * X::ROWB);
         const int64_t row = rg * CPW + grp;
         const bool rv = row < batch;
-        // ---- gather: 16-bit alpha|beta<<8 pairs and p bytes, lane totals
-        uint32_t abp[E / 2], pw[E / 4];
-        uint32_t tA = 0, tB = 0, tP = 0;
         const uint32_t seg_addr = srow + (uint32_t)(l * CPS * 16);
         const int nfull = rv ? nfull_lane : 0;  // chunks of own segment wholly before n
         if constexpr (TAIL) {
@@ -218,125 +265,205 @@ __global__ void __launch_bounds__(W * 32, 1) eval2_cdd_kernel(
             }
             __syncwarp();
         }
+        if constexpr (UCD) {
+            // ---- gather: 16-bit alpha|beta<<8 pairs, gamma pairs, M and X bytes, lane totals
+            uint32_t abp[E / 2], gp[E / 2], mw[E / 4], xw[E / 4];
+            uint32_t tA = 0, tB = 0;
 #pragma unroll
-        for (int c = 0; c < CPS; ++c) {
-            uint4 q = lds128(seg_addr + (((uint32_t)c ^ sw_own) << 4));
-            // chunks wholly past n hold the sentinel (written once, never copied over)
-            if (c < nfull) vmax = __vimax3_u16x2(__vimax3_u16x2(vmax, q.x, q.y), q.z, q.w);
-            const uint32_t wv[4] = {q.x, q.y, q.z, q.w};
-            uint32_t r[8];
+            for (int c = 0; c < CPS; ++c) {
+                uint4 q = lds128(seg_addr + (((uint32_t)c ^ sw_own) << 4));
+                if (c < nfull) vmax = __vimax3_u16x2(__vimax3_u16x2(vmax, q.x, q.y), q.z, q.w);
+                const uint32_t wv[4] = {q.x, q.y, q.z, q.w};
+                uint2 r[8];
 #pragma unroll
-            for (int j = 0; j < 4; ++j) {
-                r[2 * j] = ldtab<TOFF>(((wv[j] << SH) & amask) | tabc);
-                r[2 * j + 1] = ldtab<TOFF>(((wv[j] >> (16 - SH)) & amask) | tabc);
-            }
-#pragma unroll
-            for (int j = 0; j < 4; ++j) {
-                const uint32_t a = __byte_perm(r[2 * j], r[2 * j + 1], 0x5410u);
-                abp[4 * c + j] = a;
-                tA = __dp4a(a, 0x00010001u, tA);
-                tB = __dp4a(a, 0x01000100u, tB);
-            }
-#pragma unroll
-            for (int h = 0; h < 2; ++h) {
-                const uint32_t p01 = __byte_perm(r[4 * h], r[4 * h + 1], 0x0062u);
-                const uint32_t p23 = __byte_perm(r[4 * h + 2], r[4 * h + 3], 0x0062u);
-                const uint32_t p4 = __byte_perm(p01, p23, 0x5410u);
-                pw[2 * c + h] = p4;
-                tP = __dp4a(p4, 0x01010101u, tP);
-            }
-        }
-        // ---- scans, boundary lanes (as gchain_eval_cdd)
-        const uint32_t tAB = tA | (tB << 16);
-        const uint32_t iP = group_incl_scan<G>(tP, 0);
-        const uint32_t iAB = group_incl_scan<G>(tAB, 0);
-        const int32_t Pb = (int32_t)(iP - tP);
-        const uint32_t ABb = iAB - tAB;
-        const int32_t Ab = (int32_t)(ABb & 0xffffu), Bb = (int32_t)(ABb >> 16);
-        const int32_t Btot = (int32_t)(__shfl_sync(kFull, iAB, G - 1, G) >> 16);
-        const bool lane_valid = l * E < n;
-        const int Lk = hibit(group_ballot<G>(lane_valid && (Ab + Bb <= Btot), gbase));
-        const int Lt = hibit(group_ballot<G>(lane_valid && (Pb <= d), gbase));
-        const int Ls = max(0, min(Lk, Lt));
-        const int32_t PbS = __shfl_sync(kFull, Pb, Ls, G);
-        const uint32_t ABbS = __shfl_sync(kFull, ABb, Ls, G);
-        const int32_t thr = Btot - (int32_t)(ABbS & 0xffffu) - (int32_t)(ABbS >> 16);
-        const uint32_t key = ((uint32_t)min(thr, 0xffff) << 16) | 0xffffu;
-        // boundary row Ls: SPR consecutive positions per lane, re-gathered through the staged ids
-        const int e0 = l * SPR;
-        uint32_t idw[(SPR + 1) / 2];
-        {
-            const uint32_t bseg = srow + (uint32_t)(Ls * CPS * 16);
-            const uint32_t bsw = X::sw(grp * G + Ls);
-            if constexpr (SPR >= 8) {
-#pragma unroll
-                for (int v = 0; v < SPR / 8; ++v) {
-                    const uint4 q = lds128(bseg + ((((uint32_t)(e0 / 8 + v)) ^ bsw) << 4));
-                    idw[4 * v] = q.x; idw[4 * v + 1] = q.y; idw[4 * v + 2] = q.z; idw[4 * v + 3] = q.w;
+                for (int j = 0; j < 4; ++j) {
+                    r[2 * j] = ldtab64<TOFF>(((wv[j] << SH) & amask) | tabc);
+                    r[2 * j + 1] = ldtab64<TOFF>(((wv[j] >> (16 - SH)) & amask) | tabc);
                 }
-            } else {
-                const uint32_t a = bseg + ((((uint32_t)(e0 / 8)) ^ bsw) << 4) + (uint32_t)((e0 % 8) * 2);
-                if constexpr (SPR == 4) {
-                    uint32_t x0, x1;
-                    asm volatile("ld.shared.v2.u32 {%0,%1}, [%2];" : "=r"(x0), "=r"(x1) : "r"(a));
-                    idw[0] = x0; idw[1] = x1;
-                } else if constexpr (SPR == 2) {
-                    idw[0] = lds32(a);
+#pragma unroll
+                for (int j = 0; j < 4; ++j) {
+                    const uint32_t a = __byte_perm(r[2 * j].x, r[2 * j + 1].x, 0x5410u);
+                    abp[4 * c + j] = a;
+                    gp[4 * c + j] = __byte_perm(r[2 * j].x, r[2 * j + 1].x, 0x7632u);
+                    tA = __dp4a(a, 0x00010001u, tA);
+                    tB = __dp4a(a, 0x01000100u, tB);
+                }
+#pragma unroll
+                for (int h = 0; h < 2; ++h) {
+                    // (M0, M1, X0, X1), (M2, M3, X2, X3) -> M quad, X quad
+                    const uint32_t mx01 = __byte_perm(r[4 * h].y, r[4 * h + 1].y, 0x5140u);
+                    const uint32_t mx23 = __byte_perm(r[4 * h + 2].y, r[4 * h + 3].y, 0x5140u);
+                    mw[2 * c + h] = __byte_perm(mx01, mx23, 0x5410u);
+                    xw[2 * c + h] = __byte_perm(mx01, mx23, 0x7632u);
+                }
+            }
+            // ---- scan, boundary lane Lk (d >= sum P: the due date sits at C_{k0}; as gchain_eval_ucddcp)
+            const uint32_t tAB = tA | (tB << 16);
+            const uint32_t iAB = group_incl_scan<G>(tAB, 0);
+            const uint32_t ABb = iAB - tAB;
+            const int32_t Ab = (int32_t)(ABb & 0xffffu), Bb = (int32_t)(ABb >> 16);
+            const int32_t Btot = (int32_t)(__shfl_sync(kFull, iAB, G - 1, G) >> 16);
+            const bool lane_valid = l * E < n;
+            const int Lk = max(0, hibit(group_ballot<G>(lane_valid && (Ab + Bb <= Btot), gbase)));
+            const uint32_t ABbS = __shfl_sync(kFull, ABb, Lk, G);
+            const int e0 = l * SPR;
+            uint32_t idw[(SPR + 1) / 2];
+            e2_row_ids<G, E, SPR>(srow + (uint32_t)(Lk * CPS * 16), X::sw(grp * G + Lk), e0, idw);
+            const int kb = Lk * E + e0;
+            uint32_t rvw[SPR], mv[SPR], xv[SPR], gv[SPR];
+            uint32_t lsum = 0;
+#pragma unroll
+            for (int i = 0; i < SPR; ++i) {
+                const uint32_t id = (i & 1) ? (idw[i >> 1] >> 16) : (idw[i >> 1] & 0xffffu);
+                const uint2 rec = (rv && kb + i < n) ? ldtab64<TOFF>(((id << SH) & amask) | tabc) : make_uint2(0u, 0u);
+                rvw[i] = __byte_perm(rec.x, 0u, 0x4140u);  // alpha | beta << 16
+                gv[i] = rec.x >> 16;
+                mv[i] = rec.y & 0xffu;
+                xv[i] = (rec.y >> 8) & 0xffu;
+                lsum += rvw[i];
+            }
+            uint32_t ex = group_incl_scan<G>(lsum, 0) - lsum;
+            // elements of row Lk at or before k0 (A_excl + B_excl <= Btot, a prefix of the row)
+            // switch from the tardy weight to the early weight
+            int32_t corr = 0;
+#pragma unroll
+            for (int i = 0; i < SPR; ++i) {
+                const int32_t wA = (int32_t)(ABbS & 0xffffu) + (int32_t)(ex & 0xffffu);
+                const int32_t Bex = (int32_t)(ABbS >> 16) + (int32_t)(ex >> 16);
+                const int32_t wB = Btot - Bex;
+                const int32_t g = (int32_t)gv[i];
+                const int32_t cc = (int32_t)mv[i] * (wA - wB) + (int32_t)xv[i] * (min(wA, g) - min(wB, g));
+                corr += (wA + Bex <= Btot) ? cc : 0;
+                ex += rvw[i];
+            }
+            __syncwarp();  // every lane is done with the stage: refill it two groups ahead
+            issue(rg + 2 * gstep, st);
+            // ---- pass: pairs of weights in 16-bit halves, w2 = base2 +- f2 (Property 2: X_j
+            // compressed iff its weight exceeds gamma_j, so the X part costs min(w, gamma))
+            const bool amode = l < Lk;
+            const uint32_t wbase = (uint32_t)(amode ? Ab : (Btot - Bb));
+            const uint32_t base2 = wbase | (wbase << 16);
+            const uint32_t sgn = amode ? 1u : 0xffffffffu;
+            const uint32_t psel = amode ? 0x4044u : 0x4144u;
+            const uint32_t wsum = amode ? 0x00010001u : 0x01000100u;
+            uint32_t s = 0, acc = 0;
+#pragma unroll
+            for (int j = 0; j < E / 2; ++j) {
+                const uint32_t f2 = s * 0x10001u + __byte_perm(abp[j], 0u, psel);
+                const uint32_t w2 = f2 * sgn + base2;
+                const uint32_t mn2 = __vminu2(w2, gp[j]);
+                if (j & 1) {
+                    acc = __dp2a_hi(w2, mw[j >> 1], acc);
+                    acc = __dp2a_hi(mn2, xw[j >> 1], acc);
                 } else {
-                    uint32_t x;
-                    asm volatile("ld.shared.u16 %0, [%1];" : "=r"(x) : "r"(a));
-                    idw[0] = x;
+                    acc = __dp2a_lo(w2, mw[j >> 1], acc);
+                    acc = __dp2a_lo(mn2, xw[j >> 1], acc);
+                }
+                s = __dp4a(abp[j], wsum, s);
+            }
+            const int32_t Z = (int32_t)gsum2<G>(acc + (uint32_t)corr);
+            if (rv && l == 0) out[row] = (int64_t)Z;
+        } else {
+            // ---- gather: 16-bit alpha|beta<<8 pairs and p bytes, lane totals
+            uint32_t abp[E / 2], pw[E / 4];
+            uint32_t tA = 0, tB = 0, tP = 0;
+#pragma unroll
+            for (int c = 0; c < CPS; ++c) {
+                uint4 q = lds128(seg_addr + (((uint32_t)c ^ sw_own) << 4));
+                // chunks wholly past n hold the sentinel (written once, never copied over)
+                if (c < nfull) vmax = __vimax3_u16x2(__vimax3_u16x2(vmax, q.x, q.y), q.z, q.w);
+                const uint32_t wv[4] = {q.x, q.y, q.z, q.w};
+                uint32_t r[8];
+#pragma unroll
+                for (int j = 0; j < 4; ++j) {
+                    r[2 * j] = ldtab<TOFF>(((wv[j] << SH) & amask) | tabc);
+                    r[2 * j + 1] = ldtab<TOFF>(((wv[j] >> (16 - SH)) & amask) | tabc);
+                }
+#pragma unroll
+                for (int j = 0; j < 4; ++j) {
+                    const uint32_t a = __byte_perm(r[2 * j], r[2 * j + 1], 0x5410u);
+                    abp[4 * c + j] = a;
+                    tA = __dp4a(a, 0x00010001u, tA);
+                    tB = __dp4a(a, 0x01000100u, tB);
+                }
+#pragma unroll
+                for (int h = 0; h < 2; ++h) {
+                    const uint32_t p01 = __byte_perm(r[4 * h], r[4 * h + 1], 0x0062u);
+                    const uint32_t p23 = __byte_perm(r[4 * h + 2], r[4 * h + 3], 0x0062u);
+                    const uint32_t p4 = __byte_perm(p01, p23, 0x5410u);
+                    pw[2 * c + h] = p4;
+                    tP = __dp4a(p4, 0x01010101u, tP);
                 }
             }
-        }
-        uint32_t v[SPR];
-        uint32_t lsum = 0;
-        const int kb = Ls * E + e0;  // sequence position of this lane's first boundary element
+            // ---- scans, boundary lanes (as gchain_eval_cdd)
+            const uint32_t tAB = tA | (tB << 16);
+            const uint32_t iP = group_incl_scan<G>(tP, 0);
+            const uint32_t iAB = group_incl_scan<G>(tAB, 0);
+            const int32_t Pb = (int32_t)(iP - tP);
+            const uint32_t ABb = iAB - tAB;
+            const int32_t Ab = (int32_t)(ABb & 0xffffu), Bb = (int32_t)(ABb >> 16);
+            const int32_t Btot = (int32_t)(__shfl_sync(kFull, iAB, G - 1, G) >> 16);
+            const bool lane_valid = l * E < n;
+            const int Lk = hibit(group_ballot<G>(lane_valid && (Ab + Bb <= Btot), gbase));
+            const int Lt = hibit(group_ballot<G>(lane_valid && (Pb <= d), gbase));
+            const int Ls = max(0, min(Lk, Lt));
+            const int32_t PbS = __shfl_sync(kFull, Pb, Ls, G);
+            const uint32_t ABbS = __shfl_sync(kFull, ABb, Ls, G);
+            const int32_t thr = Btot - (int32_t)(ABbS & 0xffffu) - (int32_t)(ABbS >> 16);
+            const uint32_t key = ((uint32_t)min(thr, 0xffff) << 16) | 0xffffu;
+            // boundary row Ls: SPR consecutive positions per lane, re-gathered through the staged ids
+            const int e0 = l * SPR;
+            uint32_t idw[(SPR + 1) / 2];
+            e2_row_ids<G, E, SPR>(srow + (uint32_t)(Ls * CPS * 16), X::sw(grp * G + Ls), e0, idw);
+            uint32_t v[SPR];
+            uint32_t lsum = 0;
+            const int kb = Ls * E + e0;  // sequence position of this lane's first boundary element
 #pragma unroll
-        for (int i = 0; i < SPR; ++i) {
-            const uint32_t id = (i & 1) ? (idw[i >> 1] >> 16) : (idw[i >> 1] & 0xffffu);
-            const uint32_t rec = (rv && kb + i < n) ? ldtab<TOFF>(((id << SH) & amask) | tabc) : 0u;
-            // p | (alpha + beta) << 16
-            v[i] = __byte_perm(rec, 0u, 0x4442u) + (__dp4a(rec, 0x00000101u, 0u) << 16);
-            lsum += v[i];
-        }
-        const uint32_t ex = group_incl_scan<G>(lsum, 0) - lsum;
-        uint32_t run = ex, cinc = 0;
-        const bool sat0 = ex <= key;
+            for (int i = 0; i < SPR; ++i) {
+                const uint32_t id = (i & 1) ? (idw[i >> 1] >> 16) : (idw[i >> 1] & 0xffffu);
+                const uint32_t rec = (rv && kb + i < n) ? ldtab<TOFF>(((id << SH) & amask) | tabc) : 0u;
+                // p | (alpha + beta) << 16
+                v[i] = __byte_perm(rec, 0u, 0x4442u) + (__dp4a(rec, 0x00000101u, 0u) << 16);
+                lsum += v[i];
+            }
+            const uint32_t ex = group_incl_scan<G>(lsum, 0) - lsum;
+            uint32_t run = ex, cinc = 0;
+            const bool sat0 = ex <= key;
 #pragma unroll
-        for (int i = 0; i < SPR; ++i) {
-            const bool sat = run <= key;
-            run += v[i];
-            cinc = sat ? run : cinc;
-        }
-        const int own = max(0, hibit(group_ballot<G>(sat0, gbase)));
-        const int32_t Ck0 = PbS + (int32_t)(__shfl_sync(kFull, cinc, own, G) & 0xffffu);
-        const int32_t Dr = ((Ls == Lk) ? min(Ck0, d) : d) - PbS;
-        int32_t corr = 0;
-        run = ex;
+            for (int i = 0; i < SPR; ++i) {
+                const bool sat = run <= key;
+                run += v[i];
+                cinc = sat ? run : cinc;
+            }
+            const int own = max(0, hibit(group_ballot<G>(sat0, gbase)));
+            const int32_t Ck0 = PbS + (int32_t)(__shfl_sync(kFull, cinc, own, G) & 0xffffu);
+            const int32_t Dr = ((Ls == Lk) ? min(Ck0, d) : d) - PbS;
+            int32_t corr = 0;
+            run = ex;
 #pragma unroll
-        for (int i = 0; i < SPR; ++i) {
-            const int32_t ci = (int32_t)(run & 0xffffu), si = (int32_t)(run >> 16);
-            corr += (si - thr) * min((int32_t)(v[i] & 0xffu), max(0, Dr - ci));
-            run += v[i];
-        }
-        __syncwarp();  // every lane is done with the stage: refill it two groups ahead
-        issue(rg + 2 * gstep, st);
-        // ---- F(C_m'): early weights left of lane Ls, tardy weights from it on
-        const bool amode = l < Ls;
-        const uint32_t psel = amode ? 0x4044u : 0x4144u;
-        const uint32_t wsum = amode ? 0x00010001u : 0x01000100u;
-        uint32_t s = 0, acc = 0;
+            for (int i = 0; i < SPR; ++i) {
+                const int32_t ci = (int32_t)(run & 0xffffu), si = (int32_t)(run >> 16);
+                corr += (si - thr) * min((int32_t)(v[i] & 0xffu), max(0, Dr - ci));
+                run += v[i];
+            }
+            __syncwarp();  // every lane is done with the stage: refill it two groups ahead
+            issue(rg + 2 * gstep, st);
+            // ---- F(C_m'): early weights left of lane Ls, tardy weights from it on
+            const bool amode = l < Ls;
+            const uint32_t psel = amode ? 0x4044u : 0x4144u;
+            const uint32_t wsum = amode ? 0x00010001u : 0x01000100u;
+            uint32_t s = 0, acc = 0;
 #pragma unroll
-        for (int j = 0; j < E / 2; ++j) {
-            const uint32_t f2 = s * 0x10001u + __byte_perm(abp[j], 0u, psel);
-            acc = (j & 1) ? __dp2a_hi(f2, pw[j >> 1], acc) : __dp2a_lo(f2, pw[j >> 1], acc);
-            s = __dp4a(abp[j], wsum, s);
+            for (int j = 0; j < E / 2; ++j) {
+                const uint32_t f2 = s * 0x10001u + __byte_perm(abp[j], 0u, psel);
+                acc = (j & 1) ? __dp2a_hi(f2, pw[j >> 1], acc) : __dp2a_lo(f2, pw[j >> 1], acc);
+                s = __dp4a(abp[j], wsum, s);
+            }
+            const int32_t base = amode ? Ab : (Btot - Bb);
+            const int32_t contrib = base * (int32_t)tP + (amode ? (int32_t)acc : -(int32_t)acc) + corr;
+            const int32_t Z = (int32_t)gsum2<G>((uint32_t)contrib);
+            if (rv && l == 0) out[row] = (int64_t)Z;
         }
-        const int32_t base = amode ? Ab : (Btot - Bb);
-        const int32_t contrib = base * (int32_t)tP + (amode ? (int32_t)acc : -(int32_t)acc) + corr;
-        const int32_t Z = (int32_t)gsum2<G>((uint32_t)contrib);
-        if (rv && l == 0) out[row] = (int64_t)Z;
     }
     asm volatile("cp.async.wait_all;" ::: "memory");
     if (bad || (vmax & 0xffffu) >= (uint32_t)n || (vmax >> 16) >= (uint32_t)n) atomicOr(err, 1);
@@ -345,18 +472,18 @@ __global__ void __launch_bounds__(W * 32, 1) eval2_cdd_kernel(
 // kc_log2 = log2 of the table copies (5: conflict free, 4, 3); W warps per CTA; TOFF != 0 puts the
 // table at the window start (needs the probed base to equal TOFF).  cudaErrorNotSupported if the
 // layout does not fit.
-template <int G, int E, int W, uint32_t TOFF>
+template <int G, int E, int W, uint32_t TOFF, bool UCD = false>
 cudaError_t launch2(const Instance& I, const int16_t* perms, int64_t ld, int64_t batch,
                     int64_t* out, cudaStream_t s, int kc_log2) {
     using X = E2<G, E>;
     if (TOFF != 0 && I.smem_base != TOFF) return cudaErrorNotSupported;
     int npow2 = 1;
     while (npow2 <= I.n) npow2 <<= 1;
-    const uint32_t tbytes = (uint32_t)npow2 * 4u << kc_log2;
+    const uint32_t tbytes = (uint32_t)npow2 * (UCD ? 8u : 4u) << kc_log2;
     const uint32_t total = TOFF ? tbytes + (uint32_t)W * 2u * X::STAGE
                                 : e2_layout(I.smem_base, tbytes, 2u * X::STAGE, W).total;
     if (total > (uint32_t)kE2MaxSmem) return cudaErrorNotSupported;
-    auto kern = (I.n % 8) ? eval2_cdd_kernel<G, E, W, TOFF, true> : eval2_cdd_kernel<G, E, W, TOFF, false>;
+    auto kern = (I.n % 8) ? eval2_kernel<G, E, W, TOFF, true, UCD> : eval2_kernel<G, E, W, TOFF, false, UCD>;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)total);
     if (e != cudaSuccess) return e;
     int sms = 148;
@@ -366,17 +493,22 @@ cudaError_t launch2(const Instance& I, const int16_t* perms, int64_t ld, int64_t
     int64_t blocks = (groups + W - 1) / W;
     if (blocks > sms) blocks = sms;
     if (blocks < 1) blocks = 1;
-    kern<<<(unsigned)blocks, W * 32, total, s>>>(I.tab_ab16, I.tab_p, I.n, npow2, kc_log2, I.d_eff,
-                                                 perms, ld, batch, out, I.err);
+    kern<<<(unsigned)blocks, W * 32, total, s>>>(I.tab_ab16, I.tab_p, I.tab_m, I.tab_x, I.tab_g, I.n,
+                                                 npow2, kc_log2, I.d_eff, perms, ld, batch, out, I.err);
     return cudaGetLastError();
 }
 
-// Most copies that fit (32, 16, 8), W = 16 warps, table aligned to its size.
-template <int G, int E>
+// Most copies that fit (32, 16, 8), W = 16 warps.  UCDDCP (8-byte entries) first tries the table
+// at the window start (no alignment gap: 16 copies fit at n = 1000), then aligned to its size.
+template <int G, int E, bool UCD = false>
 cudaError_t launch2_auto(const Instance& I, const int16_t* perms, int64_t ld, int64_t batch,
                          int64_t* out, cudaStream_t s) {
     for (int kc = 5; kc >= 3; --kc) {
-        const cudaError_t e = launch2<G, E, 16, 0>(I, perms, ld, batch, out, s, kc);
+        if constexpr (UCD) {
+            const cudaError_t e = launch2<G, E, 16, 1024, true>(I, perms, ld, batch, out, s, kc);
+            if (e != cudaErrorNotSupported) return e;
+        }
+        const cudaError_t e = launch2<G, E, 16, 0, UCD>(I, perms, ld, batch, out, s, kc);
         if (e != cudaErrorNotSupported) return e;
     }
     return cudaErrorNotSupported;
@@ -421,6 +553,21 @@ cudaError_t launch_eval2_cdd(const Instance& I, const int16_t* perms, int64_t ld
     if (n <= 256) return launch2_auto<8, 32>(I, perms, ld, batch, out, s);
     if (n <= 512) return launch2_auto<8, 64>(I, perms, ld, batch, out, s);
     return launch2_auto<16, 64>(I, perms, ld, batch, out, s);
+}
+
+// UCDDCP: at most 32 positions per lane (four register arrays: alpha|beta pairs, gamma pairs,
+// M and X bytes).
+cudaError_t launch_eval2_ucddcp(const Instance& I, const int16_t* perms, int64_t ld, int64_t batch,
+                                int64_t* out, cudaStream_t s) {
+    if (!I.ab16_ok || !I.has_ucd || ld % 8 != 0 || (reinterpret_cast<uintptr_t>(perms) & 15) != 0)
+        return cudaErrorNotSupported;
+    const int n = I.n;
+    if (n <= 16 || getenv("CDD_EVAL2_NO_UCD")) return cudaErrorNotSupported;
+    if (n <= 64) return launch2_auto<4, 16, true>(I, perms, ld, batch, out, s);
+    if (n <= 128) return launch2_auto<8, 16, true>(I, perms, ld, batch, out, s);
+    if (n <= 256) return launch2_auto<8, 32, true>(I, perms, ld, batch, out, s);
+    if (n <= 512) return launch2_auto<16, 32, true>(I, perms, ld, batch, out, s);
+    return launch2_auto<32, 32, true>(I, perms, ld, batch, out, s);
 }
 
 }  // namespace cdd

@@ -57,6 +57,8 @@ cudaError_t launch_eval_batch(const Instance& I, bool ucd, const int16_t* perms,
 // layout does not apply (alpha or beta > 255, ld % 8 != 0, rows not 16-byte aligned)
 cudaError_t launch_eval2_cdd(const Instance& I, const int16_t* perms, int64_t ld, int64_t batch,
                              int64_t* out, cudaStream_t s);
+cudaError_t launch_eval2_ucddcp(const Instance& I, const int16_t* perms, int64_t ld, int64_t batch,
+                                int64_t* out, cudaStream_t s);
 cudaError_t probe_smem_base(uint32_t* base);
 
 // ---- launchers (schedule.cu) ----

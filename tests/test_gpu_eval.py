@@ -84,6 +84,36 @@ def test_ucddcp_random(lib, n):
                               _oracle(inst, perms, "ucddcp", d=d)), (n, extra)
 
 
+@pytest.mark.parametrize("n", [17, 33, 64, 65, 100, 128, 129, 200, 256, 257, 300, 512, 513, 777,
+                               999, 1000, 1023, 1024])
+@pytest.mark.parametrize("pad", [0, 5, 8])
+def test_ucddcp_batched_layouts(lib, n, pad):
+    # ucddcp_eval_batch's several-sequences-per-warp kernel (8-byte table entries): every lane
+    # layout, ragged tails (n % 8 != 0: the straddling chunk is patched in place) and garbage past
+    # n; ld % 8 != 0 takes the warp-per-sequence kernel
+    inst = gen.ucddcp_instance(n, 3 + n % 4)
+    ld = gen.pad_ld(n) + pad
+    perms = gen.random_perms(257, n, 500 + n + pad, ld=ld)
+    perms[:, n:] = 4321
+    for extra in (0, 1000):
+        d = inst.sum_p + extra
+        assert np.array_equal(_gpu_eval(lib, inst, perms, "ucddcp", d=d),
+                              _oracle(inst, perms, "ucddcp", d=d)), (n, ld, extra)
+
+
+@pytest.mark.parametrize("n", [20, 40, 300, 1000])
+def test_ucddcp_wide_values(lib, n):
+    # zero penalties, gamma = 0 and gamma up to the packed-record limit (127 with alpha, beta <= 7,
+    # p <= 30): compression decisions on both sides of min(w, gamma)
+    import dataclasses
+
+    inst = gen.ranged_instance(n, 17, (1, 30), (0, 7), (0, 7), 1.0, problem="ucddcp")
+    gamma = gen._uniform_int(gen._words(5, n, 26, n), 0, 127).astype(np.int32)
+    inst = dataclasses.replace(inst, gamma=gamma)
+    perms = gen.random_perms(300, n, n)
+    assert np.array_equal(_gpu_eval(lib, inst, perms, "ucddcp"), _oracle(inst, perms, "ucddcp"))
+
+
 def test_small_value_instances_and_zero_weights(lib):
     # tiny values, zero penalties, restrictive and unrestricted due dates
     for c in range(300):
