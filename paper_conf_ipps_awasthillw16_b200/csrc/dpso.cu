@@ -25,6 +25,10 @@ namespace {
 
 constexpr int kDpWarps = 8;
 constexpr int kDpThreads = kDpWarps * 32;
+// resident CTAs per SM the iteration kernel is compiled for (registers: 3 -> 80, 4 -> 64, 5 -> 48)
+#ifndef CDD_DP_MINB
+#define CDD_DP_MINB 3
+#endif
 
 struct DpArgs {
     ChainTables T;
@@ -269,7 +273,7 @@ __device__ __forceinline__ void fill_from(uint16_t* ids, uint16_t* inv, const in
 
 // Lines 6-7 of iteration t, then lines 4-5 of iteration t+1.
 template <int E, bool UCD, bool FAST>
-__global__ void __launch_bounds__(kDpThreads) dpso_iter_kernel(DpArgs a, int64_t t) {
+__global__ void __launch_bounds__(kDpThreads, CDD_DP_MINB) dpso_iter_kernel(DpArgs a, int64_t t) {
     using C = Chain<E, UCD>;
     constexpr int NP = C::NP;
     extern __shared__ __align__(16) uint8_t smem[];
