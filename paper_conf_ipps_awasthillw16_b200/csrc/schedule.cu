@@ -81,7 +81,7 @@ __host__ __device__ inline SchedLayout sched_layout(int n, bool ucd, int warps) 
 constexpr int kSchedWarps = 4;
 
 template <bool UCD, int E>
-__global__ void __launch_bounds__(kSchedWarps * 32) schedule_kernel(SchedArgs a) {
+__global__ void __launch_bounds__(kSchedWarps * 32, 4) schedule_kernel(SchedArgs a) {
     extern __shared__ __align__(16) uint8_t smem[];
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
     const int n = a.n;
@@ -121,16 +121,68 @@ __global__ void __launch_bounds__(kSchedWarps * 32) schedule_kernel(SchedArgs a)
     int32_t* myX = X_s + lane * CS;
     const int64_t warps = (int64_t)gridDim.x * kSchedWarps;
     bool bad = false;
-    for (int64_t row = (int64_t)blockIdx.x * kSchedWarps + wib; row < a.batch; row += warps) {
-        const int16_t* rp = a.perms + row * a.ld;
-        // ids, coalesced, validated (an id outside [0, n) raises the flag and reads job 0)
-        for (int k = lane; k < n; k += 32) {
-            const int id = rp[k];
-            const bool ok = id >= 0 && id < n;
-            bad |= !ok;
-            ids_s[(k >> lE) * IS + (k & (E - 1))] = (uint16_t)(ok ? id : 0);
+    // pairs of positions per store when rows of C (and X) are 16-byte aligned
+    const bool pairs = E >= 2 && n % 2 == 0 && (reinterpret_cast<uintptr_t>(a.C) & 15u) == 0 &&
+                       (!UCD || (reinterpret_cast<uintptr_t>(a.X) & 7u) == 0);
+    // Vector path (16-byte aligned rows, ld % 8 == 0, E >= 8): a row's ids arrive as 16-byte
+    // chunks of 8 (lane L takes chunks L, L + 32, ...) that are loaded one row AHEAD into registers,
+    // so their latency hides behind the current row's compute; each chunk lands in one lane segment.
+    constexpr int NPRE = E >= 8 ? E / 8 : 1;
+    const bool vec = E >= 8 && a.ld % 8 == 0 && (reinterpret_cast<uintptr_t>(a.perms) & 15u) == 0;
+    const int nch = (n + 7) / 8;
+    int4 pre[NPRE];
+    auto prefetch = [&](int64_t r) {
+        if (r < a.batch) {
+            const int4* src = reinterpret_cast<const int4*>(a.perms + r * a.ld);
+#pragma unroll
+            for (int t = 0; t < NPRE; ++t)
+                if (lane + 32 * t < nch) pre[t] = __ldcs(src + lane + 32 * t);
         }
-        __syncwarp();
+    };
+    const int64_t row0 = (int64_t)blockIdx.x * kSchedWarps + wib;
+    if (vec) prefetch(row0);
+    for (int64_t row = row0; row < a.batch; row += warps) {
+        const int16_t* rp = a.perms + row * a.ld;
+        if (vec) {
+#pragma unroll
+            for (int t = 0; t < NPRE; ++t) {
+                const int c = lane + 32 * t;
+                if (c < nch) {
+                    const uint32_t w[4] = {(uint32_t)pre[t].x, (uint32_t)pre[t].y, (uint32_t)pre[t].z,
+                                           (uint32_t)pre[t].w};
+                    uint32_t o[4];
+#pragma unroll
+                    for (int h = 0; h < 4; ++h) {
+                        uint32_t id2[2] = {w[h] & 0xffffu, w[h] >> 16};
+#pragma unroll
+                        for (int u = 0; u < 2; ++u) {
+                            const int k = 8 * c + 2 * h + u;
+                            if (k >= n) {
+                                id2[u] = N;  // the caller's padding: sentinel
+                            } else if (id2[u] >= N) {  // an id outside [0, n) (incl. negative)
+                                bad = true;
+                                id2[u] = 0u;
+                            }
+                        }
+                        o[h] = id2[0] | (id2[1] << 16);
+                    }
+                    const int k = 8 * c;
+                    *reinterpret_cast<uint4*>(ids_s + (k >> lE) * IS + (k & (E - 1))) =
+                        make_uint4(o[0], o[1], o[2], o[3]);
+                }
+            }
+            __syncwarp();
+            prefetch(row + warps);
+        } else {
+            // ids, coalesced, validated (an id outside [0, n) raises the flag and reads job 0)
+            for (int k = lane; k < n; k += 32) {
+                const int id = rp[k];
+                const bool ok = id >= 0 && id < n;
+                bad |= !ok;
+                ids_s[(k >> lE) * IS + (k & (E - 1))] = (uint16_t)(ok ? id : 0);
+            }
+            __syncwarp();
+        }
         // lane totals, then exclusive bases
         int32_t tP = 0, tA = 0, tB = 0;
         #pragma unroll
@@ -232,10 +284,24 @@ __global__ void __launch_bounds__(kSchedWarps * 32) schedule_kernel(SchedArgs a)
         __syncwarp();
         // coalesced copy-out of the staged rows
         int64_t* Crow = a.C + row * (int64_t)n;
-        for (int k = lane; k < n; k += 32) Crow[k] = C_s[(k >> lE) * CS + (k & (E - 1))];
+        if (pairs) {  // 16-byte streaming stores of position pairs (same lane segment: E even)
+            for (int k = 2 * lane; k < n; k += 64) {
+                const int idx = (k >> lE) * CS + (k & (E - 1));
+                __stcs(reinterpret_cast<longlong2*>(Crow + k), make_longlong2(C_s[idx], C_s[idx + 1]));
+            }
+        } else {
+            for (int k = lane; k < n; k += 32) Crow[k] = C_s[(k >> lE) * CS + (k & (E - 1))];
+        }
         if constexpr (UCD) {
             int32_t* Xrow = a.X + row * (int64_t)n;
-            for (int k = lane; k < n; k += 32) Xrow[k] = X_s[(k >> lE) * CS + (k & (E - 1))];
+            if (pairs) {
+                for (int k = 2 * lane; k < n; k += 64) {
+                    const int idx = (k >> lE) * CS + (k & (E - 1));
+                    __stcs(reinterpret_cast<int2*>(Xrow + k), make_int2(X_s[idx], X_s[idx + 1]));
+                }
+            } else {
+                for (int k = lane; k < n; k += 32) Xrow[k] = X_s[(k >> lE) * CS + (k & (E - 1))];
+            }
         }
         __syncwarp();
     }

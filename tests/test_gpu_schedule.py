@@ -95,3 +95,35 @@ def test_schedule_table1_example(lib):
     assert z == 81
     golden = oracle.cdd_eval(oracle.Problem.from_instance(inst), np.arange(5, dtype=np.int16), walk=True)[1]
     assert start == golden["s"] and np.array_equal(C, golden["C"])
+
+
+@pytest.mark.parametrize("n,pad", [(257, 7), (333, 3), (512, 0), (999, 9), (1000, 8), (1001, 7)])
+def test_schedule_vector_path_padding_and_bad_ids(lib, n, pad):
+    # n > 256 stages the ids by 16-byte chunks loaded one row ahead: garbage in the caller's padding
+    # past n is ignored, odd n stores C one position at a time, out-of-range ids raise the flag
+    import torch
+
+    inst = gen.cdd_instance(n, 9, 0.4)
+    ins = lib.Instance.from_gen(inst)
+    perms = gen.random_perms(70, n, seed=n + pad, ld=gen.pad_ld(n) + (8 if pad else 0))
+    perms[:, n:] = 4321
+    out = lib.cdd_schedule_batch(ins, torch.from_numpy(perms).cuda())
+    pen = out["penalty"].cpu().numpy()
+    C = out["C"].cpu().numpy()
+    assert np.array_equal(pen, _oracle_pens(inst, perms, n))
+    P = inst.P.astype(np.int64)
+    for r in range(0, 70, 7):
+        perm = perms[r, :n].astype(np.int64)
+        assert np.array_equal(np.diff(C[r]), P[perm][1:]), r
+        assert _cost(inst, perm, C[r], None, inst.d) == pen[r], r
+    lib.cdd_check(ins)
+    q = perms.copy()
+    q[69, n - 1] = n  # last row, last position (the straddling chunk when n % 8 != 0)
+    lib.cdd_schedule_batch(ins, torch.from_numpy(q).cuda())
+    with pytest.raises(lib.CddError):
+        lib.cdd_check(ins)
+
+
+def _oracle_pens(inst, perms, n):
+    pr = oracle.Problem.from_instance(inst)
+    return oracle.eval_batch_threaded(pr, perms, oracle.CDD)
