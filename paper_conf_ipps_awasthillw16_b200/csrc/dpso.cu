@@ -43,7 +43,7 @@ struct DpArgs {
     int32_t* zb;                   // [N]
     unsigned long long* gkey;      // [2]
     int16_t* gperm;                // [2][NP]
-    unsigned int* counter;         // [1]
+    unsigned int* counter;         // [3]: CTA arrivals, then the work counters of even / odd iterations
     int64_t* trace;
     int np;
 };
@@ -93,7 +93,10 @@ __device__ __forceinline__ void publish(const DpArgs& a, unsigned long long wkey
         const int16_t* src = a.pb + (size_t)li * a.np;
         for (int i = threadIdx.x; i < a.np; i += blockDim.x) a.gperm[(size_t)nxt * a.np + i] = src[i];
         if (threadIdx.x == 0) {
-            if (rearm) a.gkey[cur] = ULLONG_MAX;
+            if (rearm) {
+                a.gkey[cur] = ULLONG_MAX;
+                a.counter[1 + cur] = 0u;  // every CTA has left its particle loop
+            }
             *a.counter = 0u;
         }
     }
@@ -227,16 +230,24 @@ __device__ __forceinline__ uint32_t warp_excl_scan(uint32_t v, int lane, uint32_
 // written, in donor order, to positions dst(0), dst(1), ... of ids[], and inv[] follows them.
 // The donor row is read with 16-byte loads issued up front (lane L holds donor positions
 // [8L + 256 r, 8L + 256 r + 8)); the rank of a kept job is a warp scan of per-lane counts.
-template <int E, class Keep, class Dst>
-__device__ __forceinline__ void fill_from(uint16_t* ids, uint16_t* inv, const int16_t* __restrict__ donor,
-                                          int n, int lane, Keep&& keep, Dst&& dst) {
-    constexpr int R = (32 * E + 255) / 256;  // 16-byte rounds per lane
-    uint4 q[R];
+template <int E>
+constexpr int kDonorRounds = (32 * E + 255) / 256;  // 16-byte rounds per lane
+
+template <int E>
+__device__ __forceinline__ void load_donor(const int16_t* __restrict__ donor, int lane,
+                                           uint4 (&q)[kDonorRounds<E>]) {
 #pragma unroll
-    for (int r = 0; r < R; ++r) {
+    for (int r = 0; r < kDonorRounds<E>; ++r) {
         const int o = 8 * lane + 256 * r;
         q[r] = o < 32 * E ? __ldg(reinterpret_cast<const uint4*>(donor + o)) : make_uint4(0, 0, 0, 0);
     }
+}
+
+// (the donor row already in registers, loaded by load_donor)
+template <int E, class Keep, class Dst>
+__device__ __forceinline__ void fill_from(uint16_t* ids, uint16_t* inv, const uint4 (&q)[kDonorRounds<E>],
+                                          int n, int lane, Keep&& keep, Dst&& dst) {
+    constexpr int R = kDonorRounds<E>;
     uint32_t km[R];
 #pragma unroll
     for (int r = 0; r < R; ++r) {
@@ -273,7 +284,7 @@ __device__ __forceinline__ void fill_from(uint16_t* ids, uint16_t* inv, const in
 
 // Lines 6-7 of iteration t, then lines 4-5 of iteration t+1.
 template <int E, bool UCD, bool FAST>
-__global__ void __launch_bounds__(kDpThreads, CDD_DP_MINB) dpso_iter_kernel(DpArgs a, int64_t t) {
+__global__ void __launch_bounds__(kDpThreads, E >= 32 ? 2 : CDD_DP_MINB) dpso_iter_kernel(DpArgs a, int64_t t) {
     using C = Chain<E, UCD>;
     constexpr int NP = C::NP;
     extern __shared__ __align__(16) uint8_t smem[];
@@ -289,9 +300,20 @@ __global__ void __launch_bounds__(kDpThreads, CDD_DP_MINB) dpso_iter_kernel(DpAr
     const int16_t* g = a.gperm + (size_t)cur * a.np;
     const int64_t total = (int64_t)gridDim.x * kDpWarps;
     unsigned long long wkey = ULLONG_MAX;
+    // the swarm best is the same for every particle of the iteration: loaded once per warp
+    uint4 qg[kDonorRounds<E>];
+    load_donor<E>(g, lane, qg);
     __syncthreads();
-    for (int64_t i = (int64_t)blockIdx.x * kDpWarps + wib; i < a.particles; i += total) {
+    // first particle of a warp by its index; for long rows (E >= 32, n > 512) the rest come from a
+    // work counter, so a warp is done only when the swarm is (particles / warps is rarely integral
+    // and a static stride leaves the last round to a fraction of the warps): n = 1000 7.7 -> 6.9 ms
+    // per 200 iterations; for short rows the atomic costs more than the imbalance (n = 100:
+    // 2.5 -> 2.9 ms), so they keep the static stride
+    for (int64_t i = (int64_t)blockIdx.x * kDpWarps + wib; i < a.particles;) {
         const uint64_t gid = a.offset + (uint64_t)i;
+        // the personal best is issued together with the position: one round trip, not two
+        uint4 qb[kDonorRounds<E>];
+        load_donor<E>(a.pb + (size_t)i * a.np, lane, qb);
         // the position to shared memory (16-byte loads) and the position of every job
         {
             const int16_t* gp = a.pos + (size_t)i * a.np;
@@ -331,7 +353,7 @@ __global__ void __launch_bounds__(kDpThreads, CDD_DP_MINB) dpso_iter_kernel(DpAr
         // first c jobs stay, the others follow in personal-best order
         if (__dmul_rn(__dadd_rn((double)a3, 0.5), u2) < a.c1) {
             const int c = 1 + (int)bnd(b0, (uint32_t)n - 1u);
-            fill_from<E>(ids, inv, a.pb + (size_t)i * a.np, n, lane, [c](int at) { return at >= c; },
+            fill_from<E>(ids, inv, qb, n, lane, [c](int at) { return at >= c; },
                          [c](int idx) { return c + idx; });
         }
         // p(t+1) = c2 (+) F3(delta, g): two-point crossover with the swarm best -- delta[q0..q1]
@@ -346,7 +368,7 @@ __global__ void __launch_bounds__(kDpThreads, CDD_DP_MINB) dpso_iter_kernel(DpAr
                 q1 = x;
             }
             const int span = q1 - q0 + 1;
-            fill_from<E>(ids, inv, g, n, lane, [q0, q1](int at) { return at < q0 || at > q1; },
+            fill_from<E>(ids, inv, qg, n, lane, [q0, q1](int at) { return at < q0 || at > q1; },
                          [q0, span](int idx) { return idx < q0 ? idx : idx + span; });
         }
         // line 7: evaluate
@@ -366,6 +388,13 @@ __global__ void __launch_bounds__(kDpThreads, CDD_DP_MINB) dpso_iter_kernel(DpAr
         }
         const unsigned long long key = ((unsigned long long)(uint32_t)best << 32) | (uint32_t)gid;
         wkey = key < wkey ? key : wkey;
+        if constexpr (E >= 32) {
+            unsigned int w = 0;
+            if (lane == 0) w = atomicAdd(a.counter + 1 + cur, 1u);
+            i = total + (int64_t)__shfl_sync(kFull, w, 0);
+        } else {
+            i += total;
+        }
         __syncwarp();
     }
     // line 5 (iteration t+1): swarm best
@@ -446,7 +475,7 @@ template <int E, bool UCD>
 cudaError_t begin_e(Instance& I, const DpsoLaunch& p, void* ws, cudaStream_t s) {
     const DpArgs a = make_args<E>(I, p, ws);
     cudaError_t e = cudaMemsetAsync(a.gkey, 0xff, 2 * sizeof(unsigned long long), s);
-    if (e == cudaSuccess) e = cudaMemsetAsync(a.counter, 0, sizeof(unsigned int), s);
+    if (e == cudaSuccess) e = cudaMemsetAsync(a.counter, 0, 3 * sizeof(unsigned int), s);
     if (e != cudaSuccess) return e;
     const size_t smem = kDpWarps * (size_t)DpSmem<E, UCD>::BYTES;
     const int blocks = grid_for(I, dpso_init_kernel<E, UCD>, smem, p.particles);
