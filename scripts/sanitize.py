@@ -20,9 +20,11 @@ for n in (7, 50, 100, 200, 500, 777, 1000):
     if n >= 2:
         cdd.dpso_run(ins, 64, 5, seed=2)
     cdd.SaSync(ins, 64, 5, 3, seed=3, t0_samples=100).run()
+    cdd.SaSync(ins, 1024, 4, 3, seed=3, t0_samples=100).run()  # group kernel + level images
     cdd.cdd_check(ins)
     u = cdd.Instance.from_gen(gen.ucddcp_instance(n, 1))
     cdd.ucddcp_eval_batch(u, perms)
+    cdd.cdd_schedule_batch(u, perms[:50], "ucddcp")
     cdd.sa_run(u, 300, 20, problem="ucddcp", seed=1, t0_samples=100)
     if n >= 2:
         cdd.dpso_run(u, 64, 5, problem="ucddcp", seed=2)
