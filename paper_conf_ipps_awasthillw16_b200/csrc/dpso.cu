@@ -43,7 +43,8 @@ struct DpArgs {
     int32_t* zb;                   // [N]
     unsigned long long* gkey;      // [2]
     int16_t* gperm;                // [2][NP]
-    unsigned int* counter;         // [3]: CTA arrivals, then the work counters of even / odd iterations
+    unsigned int* counter;         // [4]: CTA arrivals, the work counters of even / odd iterations,
+                                   // the number of completed iterations (persistent kernel)
     int64_t* trace;
     int np;
 };
@@ -70,7 +71,7 @@ __device__ __forceinline__ void copy_out(int16_t* dst, const uint16_t* ids, int 
 // winning personal best into gperm[nxt] (and re-arms gkey[cur] for iteration t+2).
 template <int E, bool UCD>
 __device__ __forceinline__ void publish(const DpArgs& a, unsigned long long wkey, int nxt, int cur,
-                                       bool rearm) {
+                                       bool rearm, uint32_t done = 0) {
     __shared__ unsigned long long s_key[kDpWarps];
     __shared__ bool s_last;
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
@@ -98,6 +99,10 @@ __device__ __forceinline__ void publish(const DpArgs& a, unsigned long long wkey
                 a.counter[1 + cur] = 0u;  // every CTA has left its particle loop
             }
             *a.counter = 0u;
+            if (done) {  // iteration done-1 complete: release the CTAs waiting for it
+                __threadfence();
+                asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(a.counter + 3), "r"(done) : "memory");
+            }
         }
     }
 }
@@ -284,7 +289,8 @@ __device__ __forceinline__ void fill_from(uint16_t* ids, uint16_t* inv, const ui
 
 // Lines 6-7 of iteration t, then lines 4-5 of iteration t+1.
 template <int E, bool UCD, bool FAST>
-__global__ void __launch_bounds__(kDpThreads, E >= 32 ? 2 : CDD_DP_MINB) dpso_iter_kernel(DpArgs a, int64_t t) {
+__global__ void __launch_bounds__(kDpThreads, E >= 32 ? 2 : CDD_DP_MINB) dpso_iter_kernel(DpArgs a, int64_t t0,
+                                                                                          int64_t t1) {
     using C = Chain<E, UCD>;
     constexpr int NP = C::NP;
     extern __shared__ __align__(16) uint8_t smem[];
@@ -295,6 +301,7 @@ __global__ void __launch_bounds__(kDpThreads, E >= 32 ? 2 : CDD_DP_MINB) dpso_it
     uint16_t* ids = ch.id();
     uint16_t* inv = reinterpret_cast<uint16_t*>(ch.ab());  // position of each job (crossovers only)
     const int n = a.n;
+  for (int64_t t = t0; t < t1; ++t) {
     const int cur = (int)(t & 1), nxt = cur ^ 1;
     if (a.trace && blockIdx.x == 0 && threadIdx.x == 0) a.trace[t] = (int64_t)(a.gkey[cur] >> 32);
     const int16_t* g = a.gperm + (size_t)cur * a.np;
@@ -398,7 +405,19 @@ __global__ void __launch_bounds__(kDpThreads, E >= 32 ? 2 : CDD_DP_MINB) dpso_it
         __syncwarp();
     }
     // line 5 (iteration t+1): swarm best
-    publish<E, UCD>(a, wkey, nxt, cur, true);
+    publish<E, UCD>(a, wkey, nxt, cur, true, (uint32_t)(t + 1));
+    // the next iteration needs the swarm best of this one: wait for the last CTA's release
+    // (the grid is co-resident: cooperative launch)
+    if (t + 1 < t1) {
+        if (threadIdx.x == 0) {
+            uint32_t v;
+            do {
+                asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(a.counter + 3) : "memory");
+            } while ((int32_t)(v - (uint32_t)(t + 1)) < 0);
+        }
+        __syncthreads();
+    }
+  }
 }
 
 __global__ void dpso_end_kernel(const unsigned long long* gkey, const int16_t* gperm, int n,
@@ -475,7 +494,7 @@ template <int E, bool UCD>
 cudaError_t begin_e(Instance& I, const DpsoLaunch& p, void* ws, cudaStream_t s) {
     const DpArgs a = make_args<E>(I, p, ws);
     cudaError_t e = cudaMemsetAsync(a.gkey, 0xff, 2 * sizeof(unsigned long long), s);
-    if (e == cudaSuccess) e = cudaMemsetAsync(a.counter, 0, 3 * sizeof(unsigned int), s);
+    if (e == cudaSuccess) e = cudaMemsetAsync(a.counter, 0, 4 * sizeof(unsigned int), s);
     if (e != cudaSuccess) return e;
     const size_t smem = kDpWarps * (size_t)DpSmem<E, UCD>::BYTES;
     const int blocks = grid_for(I, dpso_init_kernel<E, UCD>, smem, p.particles);
@@ -493,12 +512,13 @@ cudaError_t iter_e(Instance& I, const DpsoLaunch& p, void* ws, int64_t t0, int64
     const bool fast = can_fast && I.ab16_ok;
     auto kern = fast ? dpso_iter_kernel<E, UCD, can_fast> : dpso_iter_kernel<E, UCD, false>;
     const int blocks = grid_for(I, kern, smem, p.particles);
-    for (int64_t t = t0; t < t1; ++t) {
-        kern<<<blocks, kDpThreads, smem, s>>>(a, t);
-        const cudaError_t e = cudaGetLastError();
-        if (e != cudaSuccess) return e;
-    }
-    return cudaSuccess;
+    if (t1 <= t0) return cudaSuccess;
+    // one persistent launch for iterations t0..t1-1: the CTAs wait for each other between
+    // iterations (Alg. 2 lines 4-5 need the whole swarm), so they must be co-resident -- a
+    // cooperative launch guarantees it (the grid is at most SMs x resident CTAs)
+    void* args[] = {const_cast<DpArgs*>(&a), &t0, &t1};
+    return cudaLaunchCooperativeKernel(reinterpret_cast<const void*>(kern), dim3(blocks), dim3(kDpThreads),
+                                       args, smem, s);
 }
 
 template <int E>
