@@ -246,6 +246,12 @@ def test_sa_layout_query(lib):
         assert g in (4, 8, 16, 32) and g * e >= n and (lanes == 0 or g == lanes)
         if chains < 1024:
             assert g == 32
+    # automatic choices measured fastest (profiles/r1_fig11_sweep_cdd_n1000.txt,
+    # profiles/r1b_fig11_sweep_cdd_n100.txt)
+    for n, chains, want in [(1000, 65536, 8), (1000, 4096, 16), (100, 65536, 4), (100, 16384, 4),
+                            (100, 4096, 8)]:
+        ins = lib.Instance.from_gen(gen.cdd_instance(n, 1, 0.4))
+        assert lib.sa_layout(ins, chains)[0] == want, (n, chains)
 
 
 def test_bench_config_sampled_parity(lib):
