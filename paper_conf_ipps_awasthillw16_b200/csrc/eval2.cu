@@ -563,6 +563,19 @@ cudaError_t launch_eval2_ucddcp(const Instance& I, const int16_t* perms, int64_t
         return cudaErrorNotSupported;
     const int n = I.n;
     if (n <= 16 || getenv("CDD_EVAL2_NO_UCD")) return cudaErrorNotSupported;
+    if (const char* cfg = getenv("CDD_EVAL2_UCD_GE")) {  // layout experiments: "G:E"
+        int g = 0, e = 0;
+        sscanf(cfg, "%d:%d", &g, &e);
+        const int ge = g * 1000 + e;
+        if (g * e >= n) {
+            if (ge == 8016) return launch2_auto<8, 16, true>(I, perms, ld, batch, out, s);
+            if (ge == 16016) return launch2_auto<16, 16, true>(I, perms, ld, batch, out, s);
+            if (ge == 8032) return launch2_auto<8, 32, true>(I, perms, ld, batch, out, s);
+            if (ge == 16032) return launch2_auto<16, 32, true>(I, perms, ld, batch, out, s);
+            if (ge == 32032) return launch2_auto<32, 32, true>(I, perms, ld, batch, out, s);
+            if (ge == 16064) return launch2_auto<16, 64, true>(I, perms, ld, batch, out, s);
+        }
+    }
     if (n <= 64) return launch2_auto<4, 16, true>(I, perms, ld, batch, out, s);
     if (n <= 128) return launch2_auto<8, 16, true>(I, perms, ld, batch, out, s);
     if (n <= 256) return launch2_auto<8, 32, true>(I, perms, ld, batch, out, s);
