@@ -30,7 +30,7 @@
 extern "C" {
 #endif
 
-#define CDD_ABI_VERSION 3
+#define CDD_ABI_VERSION 4
 
 #if defined(__GNUC__)
 #define CDD_API __attribute__((visibility("default")))
@@ -245,6 +245,36 @@ CDD_API int dpso_gbest_ptrs(const cdd_instance *inst, const dpso_params *params,
                     int64_t t, int64_t **key_dev, int16_t **perm_dev);
 CDD_API int dpso_end(cdd_instance *inst, const dpso_params *params, void *workspace,
              size_t workspace_bytes, void *stream);
+
+/* Fused swarm-best exchange over peer memory (one process per GPU; NVLink / NVSwitch P2P).
+ * Alg. 2 line 5 takes the swarm best over ALL particles every iteration (reading R16).
+ * Instead of two collectives between launches (dpso_gbest_ptrs + NCCL), dpso_run_peer does the
+ * exchange inside its kernels: each rank's last CTA publishes its device-local best sequence in
+ * its own region, MIN-reduces the packed key into rank 0's region with a system-scope atomic,
+ * arrives on rank 0's counter, waits for every rank, and copies the owner's sequence with peer
+ * loads.  Protocol:
+ *   dpso_peer_create(world, rank, handle): allocates this rank's region (library-owned, one
+ *       device allocation of 64 + 4 * 32 * ceil-pow2(n / 32) bytes) and returns its CUDA IPC handle
+ *       (CDD_IPC_HANDLE_BYTES bytes, written to `ipc_handle`);
+ *   the caller exchanges the handles (e.g. torch.distributed all_gather) so every rank holds all
+ *       of them in rank order;
+ *   dpso_peer_open(handles [world * CDD_IPC_HANDLE_BYTES]): maps every other rank's region;
+ *   dpso_peer_reset(stream): re-arms this rank's region -- before EVERY run, followed by a
+ *       cross-process barrier after the stream has completed (no rank may start before rank 0's
+ *       region is re-armed);
+ *   dpso_run_peer(params): the whole run (as dpso_run) with particle_offset = rank * particles
+ *       (equal shares); every rank must call it (the kernels wait for each other: all ranks'
+ *       kernels must be able to run concurrently -- one GPU per rank, or time-sliced processes);
+ *   dpso_peer_destroy: unmaps and frees (also done by cdd_instance_destroy).
+ * Results are identical to one GPU running all particles (same Philox streams, same ties).
+ * CDD_ESTATE on a wrong order of calls; CDD_ECUDA if IPC is unavailable. */
+#define CDD_IPC_HANDLE_BYTES 64
+CDD_API int dpso_peer_create(cdd_instance *inst, int world, int rank, uint8_t *ipc_handle);
+CDD_API int dpso_peer_open(cdd_instance *inst, const uint8_t *handles);
+CDD_API int dpso_peer_reset(cdd_instance *inst, void *stream);
+CDD_API int dpso_peer_destroy(cdd_instance *inst);
+CDD_API int dpso_run_peer(cdd_instance *inst, const dpso_params *params, void *workspace,
+                  size_t workspace_bytes, void *stream);
 
 /* ------------------------------------------------------------------------------------------ */
 /* Best result of the last run (SA or DPSO) on this instance                                   */

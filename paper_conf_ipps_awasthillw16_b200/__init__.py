@@ -84,6 +84,11 @@ _SIGS = {
     "dpso_iterate": (C.c_int, [_vp, C.POINTER(DpsoParams), _vp, _sz, _i64, _vp]),
     "dpso_gbest_ptrs": (C.c_int, [_vp, C.POINTER(DpsoParams), _vp, _i64, _vp, _vp]),
     "dpso_end": (C.c_int, [_vp, C.POINTER(DpsoParams), _vp, _sz, _vp]),
+    "dpso_peer_create": (C.c_int, [_vp, C.c_int, C.c_int, _vp]),
+    "dpso_peer_open": (C.c_int, [_vp, _vp]),
+    "dpso_peer_reset": (C.c_int, [_vp, _vp]),
+    "dpso_peer_destroy": (C.c_int, [_vp]),
+    "dpso_run_peer": (C.c_int, [_vp, C.POINTER(DpsoParams), _vp, _sz, _vp]),
     "best_device_ptrs": (C.c_int, [_vp, _vp, _vp]),
     "best_get": (C.c_int, [_vp, _vp, _vp, _vp, _vp]),
     "cdd_last_error": (C.c_char_p, []),
@@ -397,6 +402,12 @@ class Dpso:
         _check(_lib.dpso_run(*self._args(), _stream(stream)))
         return self
 
+    def run_peer(self, stream=None):
+        """The whole run with the swarm best exchanged inside the kernels through the instance's
+        peer exchange (dpso_peer_create / open / reset; see dist.dpso_run_distributed)."""
+        _check(_lib.dpso_run_peer(*self._args(), _stream(stream)))
+        return self
+
     def begin(self, stream=None):
         _check(_lib.dpso_begin(*self._args(), _stream(stream)))
 
@@ -425,6 +436,31 @@ def dpso_run(inst: Instance, particles: int, iters: int, problem="cdd", w=0.5, c
     """Discrete PSO (Alg. 2, eq. (3)) on one GPU; best into the instance's best buffers."""
     sw = Dpso(inst, particles, iters, problem, w, c1, c2, seed, 0, trace).run(stream)
     return {"gbest_trace": sw.trace, "workspace": sw.ws, "swarm": sw}
+
+
+IPC_HANDLE_BYTES = 64
+
+
+def dpso_peer_create(inst: Instance, world: int, rank: int) -> bytes:
+    """This rank's exchange region; returns its CUDA IPC handle (IPC_HANDLE_BYTES bytes)."""
+    h = (C.c_uint8 * IPC_HANDLE_BYTES)()
+    _check(_lib.dpso_peer_create(inst.handle, int(world), int(rank), h))
+    return bytes(h)
+
+
+def dpso_peer_open(inst: Instance, handles: list) -> None:
+    """Map every other rank's region (handles in rank order)."""
+    buf = b"".join(handles)
+    arr = (C.c_uint8 * len(buf)).from_buffer_copy(buf)
+    _check(_lib.dpso_peer_open(inst.handle, arr))
+
+
+def dpso_peer_reset(inst: Instance, stream=None) -> None:
+    _check(_lib.dpso_peer_reset(inst.handle, _stream(stream)))
+
+
+def dpso_peer_destroy(inst: Instance) -> None:
+    _check(_lib.dpso_peer_destroy(inst.handle))
 
 
 def best_device_ptrs(inst: Instance):

@@ -72,6 +72,13 @@ void free_instance(cdd_instance* I) {
     cudaFree(I->best_perm);
     cudaFree(I->stage_perm);
     cudaFree(I->stage_out);
+    if (I->peer) {
+        for (uint8_t* m : I->peer->mapped)
+            if (m) cudaIpcCloseMemHandle(m);
+        cudaFree(I->peer->d_regions);
+        cudaFree(I->peer->region);
+        delete I->peer;
+    }
     delete I;
 }
 
@@ -582,6 +589,116 @@ int dpso_end(cdd_instance* I, const dpso_params* p, void* ws, size_t ws_bytes, v
     DeviceGuard g(I->device);
     cudaError_t e = cdd::dpso_end(*I, L, ws, as_stream(stream));
     if (e != cudaSuccess) return cuda_fail(e, "dpso_end");
+    I->has_best = true;
+    return CDD_OK;
+}
+
+// ---- fused DPSO swarm-best exchange over peer memory
+int dpso_peer_create(cdd_instance* I, int world, int rank, uint8_t* ipc_handle) {
+    if (!I || !ipc_handle) return fail(CDD_EINVAL, "instance/ipc_handle is NULL");
+    if (world < 1 || rank < 0 || rank >= world) return fail(CDD_EINVAL, "need 0 <= rank < world");
+    if (I->peer) return fail(CDD_ESTATE, "a peer exchange exists on this instance (dpso_peer_destroy first)");
+    DeviceGuard g(I->device);
+    auto* P = new cdd::DpsoPeer();
+    P->world = world;
+    P->rank = rank;
+    P->np = 32 * cdd::sa_e_for_n(I->n);
+    const size_t bytes = cdd::dpso_peer_region_bytes(I->n);
+    cudaError_t e = cudaMalloc(&P->region, bytes);
+    if (e == cudaSuccess) e = cudaMemset(P->region, 0, bytes);
+    cudaIpcMemHandle_t h{};
+    if (e == cudaSuccess) e = cudaIpcGetMemHandle(&h, P->region);
+    if (e != cudaSuccess) {
+        cudaFree(P->region);
+        delete P;
+        return cuda_fail(e, "dpso_peer_create");
+    }
+    static_assert(sizeof(cudaIpcMemHandle_t) == CDD_IPC_HANDLE_BYTES, "IPC handle size");
+    std::memcpy(ipc_handle, &h, sizeof(h));
+    P->mapped.assign((size_t)world, nullptr);
+    I->peer = P;
+    return CDD_OK;
+}
+
+int dpso_peer_open(cdd_instance* I, const uint8_t* handles) {
+    if (!I || !handles) return fail(CDD_EINVAL, "instance/handles is NULL");
+    cdd::DpsoPeer* P = I->peer;
+    if (!P) return fail(CDD_ESTATE, "no peer exchange (dpso_peer_create first)");
+    if (P->open) return fail(CDD_ESTATE, "peer exchange already open");
+    DeviceGuard g(I->device);
+    std::vector<uint8_t*> regions((size_t)P->world, nullptr);
+    cudaError_t e = cudaSuccess;
+    for (int r = 0; r < P->world && e == cudaSuccess; ++r) {
+        if (r == P->rank) {
+            regions[r] = P->region;
+            continue;
+        }
+        cudaIpcMemHandle_t h{};
+        std::memcpy(&h, handles + (size_t)r * CDD_IPC_HANDLE_BYTES, sizeof(h));
+        void* ptr = nullptr;
+        e = cudaIpcOpenMemHandle(&ptr, h, cudaIpcMemLazyEnablePeerAccess);
+        P->mapped[r] = static_cast<uint8_t*>(ptr);
+        regions[r] = P->mapped[r];
+    }
+    if (e == cudaSuccess) e = cudaMalloc(&P->d_regions, sizeof(uint8_t*) * (size_t)P->world);
+    if (e == cudaSuccess)
+        e = cudaMemcpy(P->d_regions, regions.data(), sizeof(uint8_t*) * (size_t)P->world, cudaMemcpyHostToDevice);
+    if (e != cudaSuccess) {
+        for (uint8_t*& m : P->mapped)
+            if (m) cudaIpcCloseMemHandle(m), m = nullptr;
+        cudaFree(P->d_regions);
+        P->d_regions = nullptr;
+        return cuda_fail(e, "dpso_peer_open");
+    }
+    P->open = true;
+    return CDD_OK;
+}
+
+__global__ void peer_reset_kernel(uint8_t* region) {
+    if (threadIdx.x < 3) reinterpret_cast<unsigned long long*>(region + cdd::kPeerKeyOff)[threadIdx.x] = ULLONG_MAX;
+    if (threadIdx.x == 3) *reinterpret_cast<unsigned int*>(region + cdd::kPeerArriveOff) = 0u;
+}
+
+int dpso_peer_reset(cdd_instance* I, void* stream) {
+    if (!I) return fail(CDD_EINVAL, "instance is NULL");
+    if (!I->peer) return fail(CDD_ESTATE, "no peer exchange (dpso_peer_create first)");
+    DeviceGuard g(I->device);
+    peer_reset_kernel<<<1, 32, 0, as_stream(stream)>>>(I->peer->region);
+    const cudaError_t e = cudaGetLastError();
+    return e == cudaSuccess ? CDD_OK : cuda_fail(e, "dpso_peer_reset");
+}
+
+int dpso_peer_destroy(cdd_instance* I) {
+    if (!I) return fail(CDD_EINVAL, "instance is NULL");
+    if (!I->peer) return CDD_OK;
+    DeviceGuard g(I->device);
+    cudaDeviceSynchronize();
+    for (uint8_t* m : I->peer->mapped)
+        if (m) cudaIpcCloseMemHandle(m);
+    cudaFree(I->peer->d_regions);
+    cudaFree(I->peer->region);
+    delete I->peer;
+    I->peer = nullptr;
+    return CDD_OK;
+}
+
+int dpso_run_peer(cdd_instance* I, const dpso_params* p, void* ws, size_t ws_bytes, void* stream) {
+    cdd::DpsoLaunch L{};
+    int rc = dpso_prepare(I, p, ws, ws_bytes, &L);
+    if (rc != CDD_OK) return rc;
+    const cdd::DpsoPeer* P = I->peer;
+    if (!P || !P->open) return fail(CDD_ESTATE, "peer exchange not open (dpso_peer_create / dpso_peer_open)");
+    if (p->particle_offset != (uint64_t)P->rank * (uint64_t)p->particles)
+        return fail(CDD_EINVAL, "particle_offset must be rank * particles (equal shares)");
+    if ((uint64_t)p->particles * (uint64_t)P->world > (1ull << 32))
+        return fail(CDD_EINVAL, "global particle ids must fit 32 bits");
+    L.peer = true;
+    DeviceGuard g(I->device);
+    cudaStream_t s = as_stream(stream);
+    cudaError_t e = cdd::dpso_begin(*I, L, ws, s);
+    if (e == cudaSuccess) e = cdd::dpso_iterate(*I, L, ws, 0, L.iters, s);
+    if (e == cudaSuccess) e = cdd::dpso_end(*I, L, ws, s);
+    if (e != cudaSuccess) return cuda_fail(e, "dpso_run_peer");
     I->has_best = true;
     return CDD_OK;
 }

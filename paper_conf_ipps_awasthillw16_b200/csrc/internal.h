@@ -4,6 +4,7 @@
 
 #include <cstddef>
 #include <cstdint>
+#include <vector>
 
 namespace cdd {
 
@@ -18,6 +19,20 @@ struct RecLayout {
 
 constexpr uint32_t kTagSaInit = 0x11u, kTagSa = 0x12u, kTagT0 = 0x13u, kTagDpsoInit = 0x21u,
                    kTagDpso = 0x22u;
+
+// Fused DPSO swarm-best exchange over peer memory (dpso_peer_*): every rank owns one region,
+// exported by CUDA IPC and mapped by every other rank (NVLink / NVSwitch P2P between GPUs).
+// Region layout: u64 key[3] (MIN slots, rank 0's are the global ones), u32 arrivals (rank 0's
+// counts the ranks through every exchange), then int16 perm[2][np] (this rank's swarm best per
+// iteration parity, read by the others when this rank owns the global best).
+constexpr size_t kPeerKeyOff = 0, kPeerArriveOff = 24, kPeerPermOff = 64;
+struct DpsoPeer {
+    int world = 0, rank = 0, np = 0;
+    uint8_t* region = nullptr;       // own region (cudaMalloc)
+    std::vector<uint8_t*> mapped;    // peers' regions opened in this process (own slot: nullptr)
+    uint8_t** d_regions = nullptr;   // device [world]: region of every rank (own included)
+    bool open = false;
+};
 
 struct Instance {
     int device = 0;
@@ -43,6 +58,7 @@ struct Instance {
     unsigned long long* best_key = nullptr;  // device packed (penalty << 32 | id)
     int16_t* best_perm = nullptr;          // device [n]
     bool has_best = false;
+    DpsoPeer* peer = nullptr;  // dpso_peer_create / open
     // host e2e staging
     int16_t* stage_perm = nullptr;
     int64_t* stage_out = nullptr;
@@ -101,7 +117,9 @@ struct DpsoLaunch {
     double w, c1, c2;
     uint64_t seed, particle_offset;
     int64_t* gbest_trace;
+    bool peer = false;  // exchange the swarm best through Instance::peer inside the kernels
 };
+size_t dpso_peer_region_bytes(int n);
 size_t dpso_workspace_bytes(const Instance& I, const DpsoLaunch& p);
 cudaError_t dpso_begin(Instance& I, const DpsoLaunch& p, void* ws, cudaStream_t s);
 // iterations t0..t1-1 of Alg. 2 (one kernel launch each)

@@ -49,17 +49,39 @@ def global_best(inst, ids_per_rank: int, group=None) -> int:
     return reduce_best(key, perm, ids_per_rank, group)
 
 
+def peer_exchange_open(inst, group=None):
+    """Create this rank's DPSO exchange region, all-gather the CUDA IPC handles over the process
+    group and map every peer's region (dpso_peer_create / dpso_peer_open)."""
+    from . import dpso_peer_create, dpso_peer_open
+
+    world, rank = dist.get_world_size(group), dist.get_rank(group)
+    mine = dpso_peer_create(inst, world, rank)
+    handles = [None] * world
+    dist.all_gather_object(handles, mine, group=group)
+    dpso_peer_open(inst, handles)
+
+
 def dpso_run_distributed(inst, particles_per_rank: int, iters: int, problem="cdd", w=0.5, c1=0.5,
-                         c2=0.5, seed=0, group=None, trace=False):
+                         c2=0.5, seed=0, group=None, trace=False, exchange="nccl"):
     """One swarm spread over all ranks (global particle ids rank*P .. rank*P+P-1).  The swarm best of
-    Alg. 2 line 5 is global every iteration: after each device-local step the packed key is
-    MIN-all-reduced and the winner's sequence delivered to every rank (reduce_best_async: no host
-    round trip, so the iterations queue back to back), then iteration t runs."""
-    from . import Dpso
+    Alg. 2 line 5 is global every iteration.
+
+    exchange="nccl": after each device-local step the packed key is MIN-all-reduced and the
+    winner's sequence delivered to every rank (reduce_best_async: no host round trip, so the
+    iterations queue back to back), then iteration t runs.
+    exchange="p2p": one launch per rank for the whole run; the exchange happens inside the kernels
+    over peer memory (dpso_run_peer; the instance must have been through peer_exchange_open)."""
+    from . import Dpso, dpso_peer_reset
 
     rank = dist.get_rank(group)
     sw = Dpso(inst, particles_per_rank, iters, problem, w, c1, c2, seed,
               particle_offset=rank * particles_per_rank, trace=trace)
+    if exchange == "p2p":
+        dpso_peer_reset(inst)
+        torch.cuda.synchronize(inst.device)
+        dist.barrier(group)  # every region re-armed before any rank's kernels start
+        sw.run_peer()
+        return sw
     sw.begin()
     for t in range(iters):
         key, perm = sw.gbest_tensors(t)

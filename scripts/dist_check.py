@@ -2,8 +2,9 @@
 CDD_DIST_BACKEND=gloo several ranks may share one GPU):
 
   * asynchronous SA sharded over ranks + dist.global_best  ==  one run of all chains;
-  * dist.dpso_run_distributed (per-iteration swarm-best exchange)  ==  one swarm of all particles
-    (best, id, sequence and the swarm-best trace);
+  * dist.dpso_run_distributed (per-iteration swarm-best exchange, NCCL/gloo between launches and
+    fused into the kernels over peer memory)  ==  one swarm of all particles (best, id, sequence
+    and the swarm-best trace);
   * dist.sa_sync_run_distributed (per-level exchange)  ==  one synchronous run of all chains
     (best penalty; R18: the chain holding a tied best may differ).
 
@@ -56,6 +57,18 @@ def main():
     want = cdd.best_get(ref)
     assert got[0] == want[0] and got[2] == want[2] and np.array_equal(got[1], want[1]), ("dpso", got, want)
     assert np.array_equal(sw.trace.cpu().numpy()[:iters], r["gbest_trace"].cpu().numpy()[:iters]), "dpso trace"
+
+    # DPSO with the exchange fused into the kernels over peer memory (CUDA IPC regions; on one
+    # GPU the ranks' kernels are time-sliced, which is slow but exercises the same protocol)
+    if os.environ.get("CDD_DIST_P2P", "1") == "1":
+        ins = cdd.Instance.from_gen(inst, device=local)
+        cdist.peer_exchange_open(ins)
+        for rep in range(2):  # the region is re-armed per run
+            sw = cdist.dpso_run_distributed(ins, P, iters, seed=22, trace=True, exchange="p2p")
+            torch.cuda.synchronize()
+            got = cdd.best_get(ins)
+            assert got[0] == want[0] and got[2] == want[2] and np.array_equal(got[1], want[1]), ("p2p", rep, got, want)
+            assert np.array_equal(sw.trace.cpu().numpy()[:iters], r["gbest_trace"].cpu().numpy()[:iters]), "p2p trace"
 
     # synchronous SA: exchange of s^min every level
     C, M, L = 96, 10, 12
