@@ -311,6 +311,10 @@ def main():
         extra["eval_batch"] = bench_eval(lib, gens[1], dev, stream, peaks)
     if rank == 0 and not args.no_configs:
         extra["other_configs"] = bench_configs(lib, dev, stream)
+    if world > 1 and not args.no_configs:
+        dm = bench_dpso_multi_gpu(lib, cdist, dev, rank, world)
+        if rank == 0:
+            extra["dpso_multi_gpu"] = dm
     e2e = None
     if not args.no_e2e:
         e2e = bench_e2e(lib, gens, chains, steps, rank, world, dev, stream, max(1, args.steps // 2))
@@ -336,6 +340,59 @@ def main():
         print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()
+
+
+def bench_dpso_multi_gpu(lib, cdist, dev, rank, world):
+    """Config 4's swarm (CDD n=500, h=0.6, 8192 particles x 200 iterations) spread over all ranks,
+    the swarm best global every iteration: exchanged by NCCL between launches, and fused into the
+    kernels over peer memory (dpso_run_peer).  Device time, max over ranks; both give the same
+    swarm (checked on the best)."""
+    import torch
+    import torch.distributed as dist
+
+    import gen
+
+    P, iters, seed = 8192 // world, 200, 0x5EED0004
+    ins = lib.Instance.from_gen(gen.cdd_instance(500, 1, 0.6), device=dev.index)
+    out = {"workload": f"config4: CDD n=500 h=0.6, DPSO {P * world} particles ({P} per GPU) x {iters} "
+                       "iterations, swarm best global every iteration", "n_gpus": world}
+
+    def timed(prep, fn):
+        prep()
+        torch.cuda.synchronize()
+        dist.barrier()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        fn()
+        e1.record()
+        torch.cuda.synchronize()
+        t = torch.tensor([e0.elapsed_time(e1)], device=dev, dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    run_nccl = lambda: cdist.dpso_run_distributed(ins, P, iters, seed=seed)  # noqa: E731
+    timed(lambda: None, run_nccl)
+    ms = timed(lambda: None, run_nccl)
+    best_nccl = lib.best_get(ins)[0]
+    out["nccl_exchange"] = {"ms": ms, "particle_evals_per_s": P * world * (iters + 1) / (ms / 1e3)}
+    ok, why = 1, ""
+    try:
+        cdist.peer_exchange_open(ins)
+    except Exception as e:  # IPC / peer access unavailable: every rank must skip the fused run
+        ok, why = 0, str(e)[:200]
+    flag = torch.tensor([ok], device=dev, dtype=torch.int32)
+    dist.all_reduce(flag, op=dist.ReduceOp.MIN)
+    if int(flag.item()) == 1:
+        sw = lib.Dpso(ins, P, iters, seed=seed, particle_offset=rank * P)
+        prep = lambda: lib.dpso_peer_reset(ins)  # noqa: E731
+        timed(prep, lambda: sw.run_peer())
+        ms = timed(prep, lambda: sw.run_peer())
+        best = lib.best_get(ins)[0]
+        out["p2p_exchange"] = {"ms": ms, "particle_evals_per_s": P * world * (iters + 1) / (ms / 1e3),
+                               "same_best_as_nccl": best == best_nccl}
+    else:
+        out["p2p_exchange"] = {"unavailable": why or "another rank could not open the peer regions"}
+    return out
 
 
 def _timed(stream, fn, reps=1):
