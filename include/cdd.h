@@ -275,6 +275,13 @@ CDD_API int dpso_peer_reset(cdd_instance *inst, void *stream);
 CDD_API int dpso_peer_destroy(cdd_instance *inst);
 CDD_API int dpso_run_peer(cdd_instance *inst, const dpso_params *params, void *workspace,
                   size_t workspace_bytes, void *stream);
+/* Synchronous SA over all ranks with the same peer exchange (after dpso_peer_open and a
+ * dpso_peer_reset + barrier per run): every level's s^min is the minimum over the
+ * chains of ALL ranks, exchanged inside the level's finalisation kernel; chain_offset must be
+ * rank * chains.  The best-ever state stays device-local (reduce it once with best_device_ptrs).
+ * Results equal one device running all chains (R18: the chain holding a tied best may differ). */
+CDD_API int sa_sync_run_peer(cdd_instance *inst, const sa_sync_params *params, void *workspace,
+                     size_t workspace_bytes, void *stream);
 
 /* ------------------------------------------------------------------------------------------ */
 /* Best result of the last run (SA or DPSO) on this instance                                   */

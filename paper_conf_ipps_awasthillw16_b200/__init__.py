@@ -89,6 +89,7 @@ _SIGS = {
     "dpso_peer_reset": (C.c_int, [_vp, _vp]),
     "dpso_peer_destroy": (C.c_int, [_vp]),
     "dpso_run_peer": (C.c_int, [_vp, C.POINTER(DpsoParams), _vp, _sz, _vp]),
+    "sa_sync_run_peer": (C.c_int, [_vp, C.POINTER(SaSyncParams), _vp, _sz, _vp]),
     "best_device_ptrs": (C.c_int, [_vp, _vp, _vp]),
     "best_get": (C.c_int, [_vp, _vp, _vp, _vp, _vp]),
     "cdd_last_error": (C.c_char_p, []),
@@ -356,6 +357,12 @@ class SaSync:
     def run(self, stream=None):
         _check(_lib.sa_sync_run(self.inst.handle, C.byref(self.p), self.ws.data_ptr(),
                                 self.ws.numel(), _stream(stream)))
+        return self
+
+    def run_peer(self, stream=None):
+        """All levels with s^min exchanged across ranks inside the kernels (sa_sync_run_peer)."""
+        _check(_lib.sa_sync_run_peer(self.inst.handle, C.byref(self.p), self.ws.data_ptr(),
+                                     self.ws.numel(), _stream(stream)))
         return self
 
     def level(self, j: int, stream=None):

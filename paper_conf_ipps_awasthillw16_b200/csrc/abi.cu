@@ -428,6 +428,27 @@ int sa_sync_level(cdd_instance* I, const sa_sync_params* q, void* ws, size_t ws_
     return CDD_OK;
 }
 
+int sa_sync_run_peer(cdd_instance* I, const sa_sync_params* q, void* ws, size_t ws_bytes, void* stream) {
+    cdd::SaLaunch L{};
+    const int rc = sync_validate(I, q, &L);
+    if (rc != CDD_OK) return rc;
+    const cdd::DpsoPeer* P = I->peer;
+    if (!P || !P->open) return fail(CDD_ESTATE, "peer exchange not open (dpso_peer_create / dpso_peer_open)");
+    if (q->chain_offset != (uint64_t)P->rank * (uint64_t)q->chains)
+        return fail(CDD_EINVAL, "chain_offset must be rank * chains (equal shares)");
+    DeviceGuard g(I->device);
+    const size_t need = cdd::sa_sync_workspace_bytes(*I, L);
+    if (!ws || ws_bytes < need)
+        return fail(CDD_ENOMEM, "workspace too small: need " + std::to_string(need) + " bytes");
+    L.peer = true;
+    for (int64_t j = 0; j < q->levels; ++j) {
+        const cudaError_t e = cdd::launch_sa_sync_level(*I, L, j, q->level_min, ws, as_stream(stream));
+        if (e != cudaSuccess) return cuda_fail(e, "sa_sync_run_peer");
+    }
+    I->has_best = true;
+    return CDD_OK;
+}
+
 int sa_sync_run(cdd_instance* I, const sa_sync_params* q, void* ws, size_t ws_bytes, void* stream) {
     for (int64_t j = 0; q && j < q->levels; ++j) {
         const int rc = sa_sync_level(I, q, ws, ws_bytes, j, stream);

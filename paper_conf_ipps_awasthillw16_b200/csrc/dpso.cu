@@ -19,6 +19,7 @@
 #include "chain.cuh"
 #include "device_common.cuh"
 #include "internal.h"
+#include "peer.cuh"
 
 namespace cdd {
 namespace {
@@ -71,67 +72,6 @@ __device__ __forceinline__ void copy_out(int16_t* dst, const uint16_t* ids, int 
         *reinterpret_cast<int4*>(dst + o) = *reinterpret_cast<const int4*>(ids + o);
 }
 
-__device__ __forceinline__ unsigned int ld_acquire_sys(const unsigned int* p) {
-    unsigned int v;
-    asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
-    return v;
-}
-__device__ __forceinline__ unsigned long long ld_acquire_sys64(const unsigned long long* p) {
-    unsigned long long v;
-    asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
-    return v;
-}
-
-// Exchange e of the swarm best across the ranks (e = 0 after the initial positions, t + 1 after
-// iteration t), run by the whole last CTA of every rank once its device-local swarm best is in
-// gkey[par] / gperm[par]: Alg. 2 line 5 over the global swarm, fused into the kernel -- peer
-// atomics and peer reads over NVLink instead of two collectives between launches.
-//  1. the local best sequence goes to this rank's region (perm[par]), where the owner of the
-//     global best will be read from;
-//  2. MIN of the packed keys into rank 0's key slot e % 3 (a system-scope atomic), then an
-//     arrival on rank 0's counter; wait until all ranks have arrived at exchange e;
-//  3. the global key decides the owner (global id / particles per rank); a rank that does not own
-//     it copies the owner's perm[par] into its gperm[par].
-// Slot reuse: rank 0 re-arms slot (e+1) % 3 before it arrives at e -- that slot was last read at
-// exchange e-2, before every rank arrived at e-1, and no rank can use it for e+1 before rank 0
-// has arrived at e.  perm[par] is rewritten at exchange e+2, after every reader has arrived at e+1.
-template <int E, bool UCD>
-__device__ void peer_exchange(const DpArgs& a, int par, uint32_t e) {
-    __shared__ unsigned long long s_gk;
-    uint8_t* root = a.pregions[0];
-    unsigned long long* rkey = reinterpret_cast<unsigned long long*>(root + kPeerKeyOff);
-    unsigned int* rarr = reinterpret_cast<unsigned int*>(root + kPeerArriveOff);
-    int16_t* mine = reinterpret_cast<int16_t*>(a.pregions[a.pr] + kPeerPermOff) + (size_t)par * a.np;
-    int16_t* gp = a.gperm + (size_t)par * a.np;
-    for (int i = threadIdx.x; i < a.np; i += blockDim.x) mine[i] = gp[i];
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        __threadfence_system();
-        if (a.pr == 0) {
-            rkey[(e + 1) % 3] = ULLONG_MAX;
-            __threadfence_system();
-        }
-        const unsigned long long k = *(volatile unsigned long long*)&a.gkey[par];
-        atomicMin_system(&rkey[e % 3], k);
-        __threadfence_system();
-        atomicAdd_system(rarr, 1u);
-        const unsigned int target = (unsigned int)a.pw * (e + 1u);
-        while ((int)(ld_acquire_sys(rarr) - target) < 0) __nanosleep(64);
-        s_gk = ld_acquire_sys64(&rkey[e % 3]);
-    }
-    __syncthreads();
-    const unsigned long long gk = s_gk;
-    const int owner = (int)((gk & 0xffffffffull) / (unsigned long long)a.pper);
-    if (owner != a.pr) {
-        const volatile int16_t* src =
-            reinterpret_cast<const int16_t*>(a.pregions[owner] + kPeerPermOff) + (size_t)par * a.np;
-        for (int i = threadIdx.x; i < a.np; i += blockDim.x) gp[i] = src[i];
-    }
-    if (threadIdx.x == 0) a.gkey[par] = gk;
-    __threadfence();
-    __syncthreads();
-}
-
 // CTA min of the warps' keys, one atomicMin per CTA, and the last CTA to finish copies the
 // winning personal best into gperm[nxt] (and re-arms gkey[cur] for iteration t+2).
 template <int E, bool UCD>
@@ -158,9 +98,14 @@ __device__ __forceinline__ void publish(const DpArgs& a, unsigned long long wkey
         const int64_t li = (int64_t)((k & 0xffffffffull) - a.offset);
         const int16_t* src = a.pb + (size_t)li * a.np;
         for (int i = threadIdx.x; i < a.np; i += blockDim.x) a.gperm[(size_t)nxt * a.np + i] = src[i];
-        if (a.pw > 1) {
+        if (a.pw > 1) {  // Alg. 2 line 5 over the global swarm (peer.cuh)
             __syncthreads();
-            peer_exchange<E, UCD>(a, nxt, done);
+            const unsigned long long local = *(volatile unsigned long long*)&a.gkey[nxt];
+            const unsigned long long gk = peer_exchange_block(a.pregions, a.pw, a.pr, a.pper, a.np, done, nxt,
+                                                              local, a.gperm + (size_t)nxt * a.np, a.np);
+            if (threadIdx.x == 0) a.gkey[nxt] = gk;
+            __threadfence();
+            __syncthreads();
         }
         if (threadIdx.x == 0) {
             if (rearm) {

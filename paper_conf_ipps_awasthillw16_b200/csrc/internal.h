@@ -97,6 +97,7 @@ struct SaLaunch {
     int32_t lanes;  // 0 automatic, 32 warp per chain, 4 / 8 / 16 group kernel
     const int16_t* init = nullptr;  // caller's initial sequences (chain c: init + c * init_ld)
     int64_t init_ld = 0;
+    bool peer = false;  // synchronous SA: s^min exchanged through Instance::peer in the finalisation
 };
 size_t sa_workspace_bytes(const Instance& I, const SaLaunch& p);
 cudaError_t launch_t0(const Instance& I, bool ucd, uint64_t seed, int64_t samples, double* T0_dev,

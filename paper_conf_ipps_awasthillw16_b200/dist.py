@@ -94,15 +94,24 @@ def dpso_run_distributed(inst, particles_per_rank: int, iters: int, problem="cdd
 
 
 def sa_sync_run_distributed(inst, chains_per_rank: int, markov_len: int, levels: int, group=None,
-                            **kw):
+                            exchange="nccl", **kw):
     """Synchronous SA over all ranks (global chain ids rank*C .. rank*C+C-1): after
-    every temperature level the minimal final state is global -- its packed key is MIN-all-reduced
-    and the state broadcast from its owner before the next level; the best-ever state is reduced
-    once at the end (global_best)."""
-    from . import SaSync
+    every temperature level the minimal final state is global -- exchange="nccl": its packed key
+    is MIN-all-reduced and the state broadcast from its owner before the next level; "p2p": the
+    level's finalisation kernel exchanges it over peer memory (sa_sync_run_peer; the instance must
+    have been through peer_exchange_open).  The best-ever state is reduced once at the end
+    (global_best)."""
+    from . import SaSync, dpso_peer_reset
 
     rank = dist.get_rank(group)
     ss = SaSync(inst, chains_per_rank, markov_len, levels, chain_offset=rank * chains_per_rank, **kw)
+    if exchange == "p2p":
+        dpso_peer_reset(inst)
+        torch.cuda.synchronize(inst.device)
+        dist.barrier(group)
+        ss.run_peer()
+        global_best(inst, chains_per_rank, group)
+        return ss
     for j in range(levels):
         ss.level(j)
         key, perm = ss.exchange_tensors()

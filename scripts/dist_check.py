@@ -77,10 +77,19 @@ def main():
     torch.cuda.synchronize()
     got = cdd.best_get(ins)
     ref = cdd.Instance.from_gen(inst, device=local)
-    cdd.SaSync(ref, world * C, M, L, seed=23, t0_samples=500).run()
+    ref_ss = cdd.SaSync(ref, world * C, M, L, seed=23, t0_samples=500).run()
     torch.cuda.synchronize()
     want = cdd.best_get(ref)
     assert got[0] == want[0], ("sync", got[0], want[0])
+    if os.environ.get("CDD_DIST_P2P", "1") == "1":  # the level exchange fused over peer memory
+        ins = cdd.Instance.from_gen(inst, device=local)
+        cdist.peer_exchange_open(ins)
+        ss = cdist.sa_sync_run_distributed(ins, C, M, L, seed=23, t0_samples=500, exchange="p2p")
+        torch.cuda.synchronize()
+        got = cdd.best_get(ins)
+        assert got[0] == want[0], ("sync p2p", got[0], want[0])
+        # every level's s^min is the global one: the level minima equal the single run's
+        assert np.array_equal(ss.level_min.cpu().numpy(), ref_ss.level_min.cpu().numpy()), "sync p2p levels"
 
     dist.barrier()
     if rank == 0:
