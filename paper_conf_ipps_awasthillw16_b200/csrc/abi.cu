@@ -3,6 +3,9 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <map>
+#include <mutex>
+#include <tuple>
 #include <climits>
 #include <cmath>
 #include <cstring>
@@ -15,6 +18,32 @@
 using cdd::Instance;
 
 struct cdd_instance : Instance {};
+
+namespace cdd {
+void resident_ctas(const void* kern, int device, int threads, size_t smem, int* sms, int* occ) {
+    static std::mutex mu;
+    static std::map<std::tuple<const void*, int, int, size_t>, std::pair<int, int>> memo;
+    const auto key = std::make_tuple(kern, device, threads, smem);
+    {
+        std::lock_guard<std::mutex> lk(mu);
+        const auto it = memo.find(key);
+        if (it != memo.end()) {
+            *sms = it->second.first;
+            *occ = it->second.second;
+            return;
+        }
+    }
+    int s = 148, o = 1;
+    cudaDeviceGetAttribute(&s, cudaDevAttrMultiProcessorCount, device);
+    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, kern, threads, smem);
+    if (o < 1) o = 1;
+    *sms = s;
+    *occ = o;
+    std::lock_guard<std::mutex> lk(mu);
+    memo[key] = {s, o};
+}
+}  // namespace cdd
 
 namespace {
 
@@ -88,6 +117,8 @@ extern "C" {
 
 const char* cdd_last_error(void) { return g_err.c_str(); }
 int cdd_abi_version(void) { return CDD_ABI_VERSION; }
+
+
 
 int cdd_instance_create(int32_t n, const int32_t* p, const int32_t* alpha, const int32_t* beta,
                         const int32_t* m, const int32_t* gamma, int64_t d, int device,

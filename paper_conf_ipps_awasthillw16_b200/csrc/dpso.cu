@@ -500,10 +500,7 @@ DpArgs make_args(const Instance& I, const DpsoLaunch& p, void* ws) {
 template <class K>
 int grid_for(const Instance& I, K kern, size_t smem, int64_t particles) {
     int sms = 148, occ = 1;
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, I.device);
-    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kDpThreads, smem);
-    if (occ < 1) occ = 1;
+    resident_ctas(reinterpret_cast<const void*>(kern), I.device, kDpThreads, smem, &sms, &occ);
     int64_t need = (particles + kDpWarps - 1) / kDpWarps;
     const int64_t cap = (int64_t)sms * occ;
     if (need > cap) need = cap;

@@ -65,6 +65,11 @@ struct Instance {
     size_t stage_rows = 0;
 };
 
+// Resident CTAs per SM of `kern` with `threads` threads and `smem` dynamic shared memory (the
+// dynamic-smem attribute is raised to `smem` first), and the device's SM count; memoised per
+// (kernel, device, threads, smem) -- the runtime queries cost more host time than a launch.
+void resident_ctas(const void* kern, int device, int threads, size_t smem, int* sms, int* occ);
+
 // ---- launchers (eval.cu) ----
 cudaError_t launch_eval_batch(const Instance& I, bool ucd, const int16_t* perms, int64_t ld,
                               int64_t batch, int64_t* out, cudaStream_t s);
