@@ -97,3 +97,55 @@ def test_dpso_n10_reaches_optimum(lib):
     lib.dpso_run(ins, 768, 200, seed=5)  # 768 particles as in the paper
     pen, perm, gid = lib.best_get(ins)
     assert pen == gold["optimum"]
+
+
+def test_peer_exchange_api_single_rank(lib):
+    # the fused-exchange entry points on one rank: argument / state errors, and a world-1 exchange
+    # (no peers) equals dpso_run and sa_sync_run exactly
+    import torch
+
+    inst = gen.cdd_instance(120, 4, 0.4)
+    ins = lib.Instance.from_gen(inst)
+    sw = lib.Dpso(ins, 96, 12, seed=5, trace=True)
+    with pytest.raises(lib.CddError) as e:
+        sw.run_peer()  # no exchange yet
+    assert e.value.code == lib.CDD_ESTATE
+    with pytest.raises(lib.CddError) as e:
+        lib.dpso_peer_create(ins, 2, 2)  # rank outside [0, world)
+    assert e.value.code == lib.CDD_EINVAL
+    h = lib.dpso_peer_create(ins, 1, 0)
+    assert len(h) == lib.IPC_HANDLE_BYTES
+    with pytest.raises(lib.CddError) as e:
+        lib.dpso_peer_create(ins, 1, 0)  # one exchange per instance
+    assert e.value.code == lib.CDD_ESTATE
+    with pytest.raises(lib.CddError) as e:
+        sw.run_peer()  # created, not open
+    assert e.value.code == lib.CDD_ESTATE
+    lib.dpso_peer_open(ins, [h])
+    lib.dpso_peer_reset(ins)
+    sw.run_peer()
+    torch.cuda.synchronize()
+    got, gtr = lib.best_get(ins), sw.trace.cpu().numpy()
+    ref = lib.Instance.from_gen(inst)
+    r = lib.dpso_run(ref, 96, 12, seed=5, trace=True)
+    torch.cuda.synchronize()
+    want = lib.best_get(ref)
+    assert got[0] == want[0] and got[2] == want[2] and np.array_equal(got[1], want[1])
+    assert np.array_equal(gtr, r["gbest_trace"].cpu().numpy())
+    bad = lib.Dpso(ins, 96, 12, seed=5, particle_offset=7)
+    with pytest.raises(lib.CddError) as e:
+        bad.run_peer()  # particle_offset must be rank * particles
+    assert e.value.code == lib.CDD_EINVAL
+    # synchronous SA through the same exchange
+    lib.dpso_peer_reset(ins)
+    ss = lib.SaSync(ins, 2048, 6, 4, seed=9, t0_samples=300).run_peer()
+    torch.cuda.synchronize()
+    s_ref = lib.SaSync(ref, 2048, 6, 4, seed=9, t0_samples=300).run()
+    torch.cuda.synchronize()
+    assert lib.best_get(ins)[0] == lib.best_get(ref)[0]
+    assert np.array_equal(ss.level_min.cpu().numpy(), s_ref.level_min.cpu().numpy())
+    lib.dpso_peer_destroy(ins)
+    with pytest.raises(lib.CddError):
+        sw.run_peer()
+    ins.destroy()
+    ref.destroy()
