@@ -49,6 +49,13 @@ def global_best(inst, ids_per_rank: int, group=None) -> int:
     return reduce_best(key, perm, ids_per_rank, group)
 
 
+def global_best_async(inst, group=None) -> None:
+    """global_best without the host round trip (reduce_best_async on the best buffers): the next
+    run's launches queue behind the collectives instead of waiting for them."""
+    key, perm = best_device_tensors(inst)
+    reduce_best_async(key, perm, group)
+
+
 def peer_exchange_open(inst, group=None):
     """Create this rank's DPSO exchange region, all-gather the CUDA IPC handles over the process
     group and map every peer's region (dpso_peer_create / dpso_peer_open)."""

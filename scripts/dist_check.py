@@ -44,6 +44,11 @@ def main():
     cdd.sa_run(ref, world * C, steps, seed=21, t0_samples=500)
     want = cdd.best_get(ref)
     assert got[0] == want[0] and got[2] == want[2] and np.array_equal(got[1], want[1]), ("sa", got, want)
+    ins = cdd.Instance.from_gen(inst, device=local)  # the same without a host round trip
+    cdd.sa_run(ins, C, steps, seed=21, t0_samples=500, chain_offset=rank * C)
+    cdist.global_best_async(ins)
+    got = cdd.best_get(ins)
+    assert got[0] == want[0] and got[2] == want[2] and np.array_equal(got[1], want[1]), ("sa async", got, want)
 
     # DPSO: one swarm over all ranks, exchange every iteration
     P, iters = 48, 25
