@@ -548,6 +548,23 @@ cudaError_t launch_eval2_cdd(const Instance& I, const int16_t* perms, int64_t ld
         return flat ? launch2<16, 64, 16, 1024>(I, perms, ld, batch, out, s, kc)
                     : launch2<16, 64, 16, 0>(I, perms, ld, batch, out, s, kc);
     }
+    if (const char* cfg = getenv("CDD_EVAL2_GE")) {  // layout experiments: "G:E"
+        int g = 0, e = 0;
+        sscanf(cfg, "%d:%d", &g, &e);
+        if (g * e >= n) {
+            switch (g * 1000 + e) {
+                case 4016: return launch2_auto<4, 16>(I, perms, ld, batch, out, s);
+                case 4032: return launch2_auto<4, 32>(I, perms, ld, batch, out, s);
+                case 8016: return launch2_auto<8, 16>(I, perms, ld, batch, out, s);
+                case 8032: return launch2_auto<8, 32>(I, perms, ld, batch, out, s);
+                case 8064: return launch2_auto<8, 64>(I, perms, ld, batch, out, s);
+                case 16016: return launch2_auto<16, 16>(I, perms, ld, batch, out, s);
+                case 16032: return launch2_auto<16, 32>(I, perms, ld, batch, out, s);
+                case 16064: return launch2_auto<16, 64>(I, perms, ld, batch, out, s);
+                default: break;
+            }
+        }
+    }
     if (n <= 64) return launch2_auto<4, 16>(I, perms, ld, batch, out, s);
     if (n <= 128) return launch2_auto<4, 32>(I, perms, ld, batch, out, s);
     if (n <= 256) return launch2_auto<8, 32>(I, perms, ld, batch, out, s);
