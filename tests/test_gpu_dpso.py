@@ -149,3 +149,21 @@ def test_peer_exchange_api_single_rank(lib):
         sw.run_peer()
     ins.destroy()
     ref.destroy()
+
+
+def test_config4_full_size_parity(lib):
+    # BASELINE config 4 exactly as bench.py launches it (CDD n=500, h=0.6, instance seed 1, 8192
+    # particles x 200 iterations, seed 0x5EED0004, one persistent launch): the oracle replays the
+    # whole swarm (~10 s) -- best value, particle id, sequence and the per-iteration swarm best
+    import torch
+
+    inst = gen.cdd_instance(500, 1, 0.6)
+    ins = lib.Instance.from_gen(inst)
+    sw = lib.Dpso(ins, 8192, 200, seed=0x5EED0004, trace=True).run()
+    torch.cuda.synchronize()
+    got = lib.best_get(ins)
+    ref = oracle.dpso_run(oracle.Problem.from_instance(inst),
+                          oracle.dpso_params(particles=8192, iters=200, seed=0x5EED0004), trace=True)
+    assert (got[0], got[2]) == (ref["E_best"], ref["id"])
+    assert np.array_equal(got[1], ref["best"])
+    assert np.array_equal(sw.trace.cpu().numpy(), ref["gbest_trace"])
