@@ -277,3 +277,44 @@ def test_bench_config_sampled_parity(lib):
     p = oracle.sa_params(chains=1, steps=bench.SA_STEPS, seed=bench.RUN_SEED)
     for c in [0, 1, 31, 4096, 40000, bench.CHAINS - 1, gid]:
         assert oracle.sa_chain(pr, p, T0v, c)["E_best"] == cb[c], c
+
+
+def test_configs_2_3_sampled_parity(lib):
+    # BASELINE configs 2 and 3 exactly as bench.py launches them (automatic layouts, T0 from 5000
+    # samples inside sa_run): config 2 = CDD n=100, instance 1, every h, 4096 chains x 5000 steps
+    # plus the 2^20-sequence batched evaluation; config 3 = UCDDCP n=200 (d = sum p), 16384 chains
+    # x 5000 steps.  The oracle recomputes T0, replays sampled chains and evaluates sampled rows.
+    import torch
+
+    p2 = gen.random_perms_device(1 << 20, 100, 2)
+    rows = [0, 1, 777, 123456, 524287, (1 << 20) - 1]
+    sample = p2[rows].cpu().numpy()
+    for h in gen.H_VALUES:
+        inst = gen.cdd_instance(100, 1, h)
+        ins = lib.Instance.from_gen(inst)
+        pr = _prob(inst)
+        z = lib.cdd_eval_batch(ins, p2).cpu().numpy()
+        assert np.array_equal(z[rows], oracle.eval_batch(pr, sample)), h
+        res = lib.sa_run(ins, 4096, 5000, seed=0x5EED0002, chain_best=True)
+        torch.cuda.synchronize()
+        T0 = float(res["T0"].item())
+        assert T0 == oracle.t0(pr, oracle.CDD, 0x5EED0002, 5000), h
+        cb = res["chain_best"].cpu().numpy()
+        pen, perm, gid = lib.best_get(ins)
+        assert pen == cb.min() and gid == int(np.argmin(cb)) and oracle.cdd_eval(pr, perm) == pen
+        p = oracle.sa_params(chains=1, steps=5000, seed=0x5EED0002)
+        for c in [0, 2049, 4095, gid]:
+            assert oracle.sa_chain(pr, p, T0, c)["E_best"] == cb[c], (h, c)
+    inst = gen.ucddcp_instance(200, 1)
+    ins = lib.Instance.from_gen(inst)
+    pr = _prob(inst)
+    res = lib.sa_run(ins, 16384, 5000, problem="ucddcp", seed=0x5EED0003, chain_best=True)
+    torch.cuda.synchronize()
+    T0 = float(res["T0"].item())
+    assert T0 == oracle.t0(pr, oracle.UCDDCP, 0x5EED0003, 5000)
+    cb = res["chain_best"].cpu().numpy()
+    pen, perm, gid = lib.best_get(ins)
+    assert pen == cb.min() and gid == int(np.argmin(cb))
+    p = oracle.sa_params(problem=oracle.UCDDCP, chains=1, steps=5000, seed=0x5EED0003)
+    for c in [0, 8191, 16383, gid]:
+        assert oracle.sa_chain(pr, p, T0, c)["E_best"] == cb[c], c
