@@ -29,5 +29,16 @@ for n in (7, 50, 100, 200, 500, 777, 1000):
     if n >= 2:
         cdd.dpso_run(u, 64, 5, problem="ucddcp", seed=2)
     cdd.cdd_check(u)
+# fused exchange entry points on one rank (world 1), T0 on the group layout via sa_t0
+ins = cdd.Instance.from_gen(gen.cdd_instance(300, 2, 0.4))
+cdd.sa_t0(ins, samples=700)
+h = cdd.dpso_peer_create(ins, 1, 0)
+cdd.dpso_peer_open(ins, [h])
+cdd.dpso_peer_reset(ins)
+cdd.Dpso(ins, 64, 4, seed=2).run_peer()
+cdd.dpso_peer_reset(ins)
+cdd.SaSync(ins, 1024, 3, 2, seed=3, t0_samples=100).run_peer()
+cdd.dpso_peer_destroy(ins)
+cdd.cdd_check(ins)
 torch.cuda.synchronize()
 print("sanitize run ok")
