@@ -29,6 +29,10 @@ for n in (7, 50, 100, 200, 500, 777, 1000):
     if n >= 2:
         cdd.dpso_run(u, 64, 5, problem="ucddcp", seed=2)
     cdd.cdd_check(u)
+# balanced SA schedule (chains split between warps, state handed over): more chains than slots
+ins = cdd.Instance.from_gen(gen.cdd_instance(120, 2, 0.4))
+cdd.sa_run(ins, 15000, 9, seed=4, T0=900.0, lanes=8)
+cdd.cdd_check(ins)
 # fused exchange entry points on one rank (world 1), T0 on the group layout via sa_t0
 ins = cdd.Instance.from_gen(gen.cdd_instance(300, 2, 0.4))
 cdd.sa_t0(ins, samples=700)

@@ -318,3 +318,36 @@ def test_configs_2_3_sampled_parity(lib):
     p = oracle.sa_params(problem=oracle.UCDDCP, chains=1, steps=5000, seed=0x5EED0003)
     for c in [0, 8191, 16383, gid]:
         assert oracle.sa_chain(pr, p, T0, c)["E_best"] == cb[c], c
+
+
+@pytest.mark.parametrize("problem,n,chains,steps", [("cdd", 200, 16000, 200), ("ucddcp", 200, 16384, 150),
+                                                    ("cdd", 120, 15000, 37)])
+def test_balanced_schedule_every_chain(lib, problem, n, chains, steps):
+    # more chains than resident slots but a mostly empty last round: the balanced schedule splits
+    # chains between two warps (state handed over mid-run); every chain's best and final penalty,
+    # the winner and its sequence must equal the oracle's replay -- and the round-robin run
+    import os
+    import torch
+
+    inst = gen.ucddcp_instance(n, 2) if problem == "ucddcp" else gen.cdd_instance(n, 2, 0.4)
+    ins = lib.Instance.from_gen(inst)
+    res = lib.sa_run(ins, chains, steps, problem=problem, seed=77, T0=2500.0, lanes=8,
+                     chain_best=True, chain_final=True)
+    torch.cuda.synchronize()
+    cb, cf = res["chain_best"].cpu().numpy(), res["chain_final"].cpu().numpy()
+    pen, perm, gid = lib.best_get(ins)
+    pr = _prob(inst)
+    code = oracle.UCDDCP if problem == "ucddcp" else oracle.CDD
+    p = oracle.sa_params(problem=code, chains=1, steps=steps, seed=77)
+    for c in range(chains):
+        r = oracle.sa_chain(pr, p, 2500.0, c)
+        assert (r["E_best"], r["E_final"]) == (cb[c], cf[c]), c
+    assert pen == cb.min() and gid == int(np.argmin(cb))
+    assert np.array_equal(perm, oracle.sa_chain(pr, p, 2500.0, gid)["best"])
+    os.environ["CDD_SA_BALANCE"] = "0"
+    try:
+        r2 = lib.sa_run(ins, chains, steps, problem=problem, seed=77, T0=2500.0, lanes=8, chain_best=True)
+        torch.cuda.synchronize()
+        assert np.array_equal(r2["chain_best"].cpu().numpy(), cb)
+    finally:
+        del os.environ["CDD_SA_BALANCE"]
