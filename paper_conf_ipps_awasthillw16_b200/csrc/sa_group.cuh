@@ -27,6 +27,10 @@
 #ifndef CDD_SAG_PREFETCH
 #define CDD_SAG_PREFETCH 0
 #endif
+// 1: the CDD pass runs the two halves of a lane row as independent dependency chains (experiment)
+#ifndef CDD_SAG_SPLITPASS
+#define CDD_SAG_SPLITPASS 0
+#endif
 
 namespace cdd {
 
@@ -338,16 +342,46 @@ __device__ __forceinline__ int32_t gchain_eval_cdd(const GChain<G, E>& ch, int l
     const uint8_t* arow = reinterpret_cast<const uint8_t*>(ch.ab()) + l * C::AS;
     const uint8_t* prow = ch.pb() + l * C::PS;
     constexpr int CH = E >= 16 ? 16 : E;  // positions per chunk
+#if CDD_SAG_SPLITPASS
+    if constexpr (E >= 2 * CH) {
+        // two independent halves (ILP 2 on the s / acc dependency chains): the second half starts
+        // from s = 0 and is corrected by s_mid * (sum of p over the second half)
+        constexpr int HALF = E / 2;
+        uint32_t s2 = 0, acc2 = 0, p2 = 0;
 #pragma unroll
-    for (int c0 = 0; c0 < E; c0 += CH) {
-        uint32_t r[CH / 2], q[CH / 4];
-        load_ab16<CH>(arow + 2 * c0, r);
-        load_b8<CH>(prow + c0, q);
+        for (int c0 = 0; c0 < HALF; c0 += CH) {
+            uint32_t r[CH / 2], q[CH / 4], rb[CH / 2], qb[CH / 4];
+            load_ab16<CH>(arow + 2 * c0, r);
+            load_b8<CH>(prow + c0, q);
+            load_ab16<CH>(arow + 2 * (c0 + HALF), rb);
+            load_b8<CH>(prow + c0 + HALF, qb);
 #pragma unroll
-        for (int j = 0; j < CH / 2; ++j) {
-            const uint32_t f2 = s * 0x10001u + __byte_perm(r[j], 0u, psel);
-            acc = (j & 1) ? __dp2a_hi(f2, q[j >> 1], acc) : __dp2a_lo(f2, q[j >> 1], acc);
-            s = __dp4a(r[j], wsum, s);
+            for (int j = 0; j < CH / 2; ++j) {
+                const uint32_t f2 = s * 0x10001u + __byte_perm(r[j], 0u, psel);
+                const uint32_t g2 = s2 * 0x10001u + __byte_perm(rb[j], 0u, psel);
+                acc = (j & 1) ? __dp2a_hi(f2, q[j >> 1], acc) : __dp2a_lo(f2, q[j >> 1], acc);
+                acc2 = (j & 1) ? __dp2a_hi(g2, qb[j >> 1], acc2) : __dp2a_lo(g2, qb[j >> 1], acc2);
+                s = __dp4a(r[j], wsum, s);
+                s2 = __dp4a(rb[j], wsum, s2);
+            }
+#pragma unroll
+            for (int j = 0; j < CH / 4; ++j) p2 = __dp4a(qb[j], 0x01010101u, p2);
+        }
+        acc += acc2 + s * p2;
+    } else
+#endif
+    {
+#pragma unroll
+        for (int c0 = 0; c0 < E; c0 += CH) {
+            uint32_t r[CH / 2], q[CH / 4];
+            load_ab16<CH>(arow + 2 * c0, r);
+            load_b8<CH>(prow + c0, q);
+#pragma unroll
+            for (int j = 0; j < CH / 2; ++j) {
+                const uint32_t f2 = s * 0x10001u + __byte_perm(r[j], 0u, psel);
+                acc = (j & 1) ? __dp2a_hi(f2, q[j >> 1], acc) : __dp2a_lo(f2, q[j >> 1], acc);
+                s = __dp4a(r[j], wsum, s);
+            }
         }
     }
 #endif
