@@ -534,8 +534,19 @@ cudaError_t iter_e(Instance& I, const DpsoLaunch& p, void* ws, int64_t t0, int64
     // iterations (Alg. 2 lines 4-5 need the whole swarm), so they must be co-resident -- a
     // cooperative launch guarantees it (the grid is at most SMs x resident CTAs)
     void* args[] = {const_cast<DpArgs*>(&a), &t0, &t1};
-    return cudaLaunchCooperativeKernel(reinterpret_cast<const void*>(kern), dim3(blocks), dim3(kDpThreads),
-                                       args, smem, s);
+    cudaError_t e = cudaLaunchCooperativeKernel(reinterpret_cast<const void*>(kern), dim3(blocks),
+                                                dim3(kDpThreads), args, smem, s);
+    if (e == cudaErrorCooperativeLaunchTooLarge || e == cudaErrorNotSupported) {
+        // co-residency not available here: one launch per iteration (no in-kernel wait)
+        (void)cudaGetLastError();
+        for (int64_t t = t0; t < t1; ++t) {
+            kern<<<blocks, kDpThreads, smem, s>>>(a, t, t + 1);
+            const cudaError_t le = cudaGetLastError();
+            if (le != cudaSuccess) return le;
+        }
+        return cudaSuccess;
+    }
+    return e;
 }
 
 template <int E>
