@@ -185,21 +185,33 @@ __global__ void __launch_bounds__(kSchedWarps * 32, 4) schedule_kernel(SchedArgs
         }
         // lane totals, then exclusive bases; the records stay in registers for the later passes
         // (the compiler cannot keep them across the shared-memory stores of C otherwise)
-        uint32_t rr[E], pq[(E + 3) / 4];
+        // (CDD only: the UCDDCP passes need more per-position data than the registers hold)
+        constexpr int RC = UCD ? 1 : E;
+        uint32_t rr[RC], pq[(RC + 3) / 4];
         #pragma unroll
-        for (int i = 0; i < (E + 3) / 4; ++i) pq[i] = 0u;
+        for (int i = 0; i < (RC + 3) / 4; ++i) pq[i] = 0u;
         int32_t tP = 0, tA = 0, tB = 0;
         #pragma unroll
         for (int i = 0; i < E; ++i) {
             const int j = myids[i];
-            rr[i] = t_ab[j];
+            const uint32_t r = t_ab[j];
             const uint32_t pj = t_p[j];
-            pq[i / 4] |= pj << (8 * (i % 4));
+            if constexpr (!UCD) {
+                rr[i] = r;
+                pq[i / 4] |= pj << (8 * (i % 4));
+            }
             tP += (int32_t)pj;
-            tA += (int32_t)(rr[i] & 0xffffu);
-            tB += (int32_t)(rr[i] >> 16);
+            tA += (int32_t)(r & 0xffffu);
+            tB += (int32_t)(r >> 16);
         }
-        auto rec_p = [&](int i) { return (int32_t)((pq[i / 4] >> (8 * (i % 4))) & 0xffu); };
+        auto rec_r = [&](int i) {
+            if constexpr (UCD) return t_ab[myids[i]];
+            else return rr[i];
+        };
+        auto rec_p = [&](int i) {
+            if constexpr (UCD) return (int32_t)t_p[myids[i]];
+            else return (int32_t)((pq[i / 4] >> (8 * (i % 4))) & 0xffu);
+        };
         const int32_t Pb = warp_excl_scan(tP, lane), Ab = warp_excl_scan(tA, lane),
                       Bb = warp_excl_scan(tB, lane);
         const int32_t Btot = __shfl_sync(kFull, Bb + tB, 31);
@@ -210,7 +222,7 @@ __global__ void __launch_bounds__(kSchedWarps * 32, 4) schedule_kernel(SchedArgs
             int32_t c = Pb, s = Ab + Bb;
             #pragma unroll
         for (int i = 0; i < E; ++i) {
-                const uint32_t r = rr[i];
+                const uint32_t r = rec_r(i);
                 c += rec_p(i);
                 if (s <= Btot) {
                     k0 = k_lo + i;
@@ -231,7 +243,7 @@ __global__ void __launch_bounds__(kSchedWarps * 32, 4) schedule_kernel(SchedArgs
             int64_t c = st + Pb;
             #pragma unroll
         for (int i = 0; i < E; ++i) {
-                const uint32_t r = rr[i];
+                const uint32_t r = rec_r(i);
                 c += rec_p(i);
                 myC[i] = c;
                 pen += (int64_t)(r & 0xffffu) * max((int64_t)0, a.d - c) +
