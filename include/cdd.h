@@ -267,6 +267,8 @@ CDD_API int dpso_end(cdd_instance *inst, const dpso_params *params, void *worksp
  *       kernels must be able to run concurrently -- one GPU per rank, or time-sliced processes);
  *   dpso_peer_destroy: unmaps and frees (also done by cdd_instance_destroy).
  * Results are identical to one GPU running all particles (same Philox streams, same ties).
+ * A rank that never arrives at an exchange (its process died) does not hang the others: after 30 s
+ * the wait gives up and cdd_check reports CDD_EDATA ("a peer rank never reached ...").
  * CDD_ESTATE on a wrong order of calls; CDD_ECUDA if IPC is unavailable. */
 #define CDD_IPC_HANDLE_BYTES 64
 CDD_API int dpso_peer_create(cdd_instance *inst, int world, int rank, uint8_t *ipc_handle);

@@ -359,7 +359,8 @@ int cdd_check(cdd_instance* I, void* stream) {
     if (flag) {
         cudaMemsetAsync(I->err, 0, sizeof(int), s);
         cudaStreamSynchronize(s);
-        return fail(CDD_EDATA, "a sequence contained a job id outside [0, n)");
+        return fail(CDD_EDATA, (flag & 2) ? "a peer rank never reached a swarm-best exchange (timed out)"
+                                          : "a sequence contained a job id outside [0, n)");
     }
     return CDD_OK;
 }

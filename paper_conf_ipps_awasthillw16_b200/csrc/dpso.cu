@@ -48,6 +48,7 @@ struct DpArgs {
     int pw, pr;
     int64_t pper;
     uint8_t* const* pregions;
+    int* err;  // instance error flag (bit 2: a peer never arrived)
     unsigned int* counter;         // [4]: CTA arrivals, the work counters of even / odd iterations,
                                    // the number of completed iterations (persistent kernel)
     int64_t* trace;
@@ -102,7 +103,7 @@ __device__ __forceinline__ void publish(const DpArgs& a, unsigned long long wkey
             __syncthreads();
             const unsigned long long local = *(volatile unsigned long long*)&a.gkey[nxt];
             const unsigned long long gk = peer_exchange_block(a.pregions, a.pw, a.pr, a.pper, a.np, done, nxt,
-                                                              local, a.gperm + (size_t)nxt * a.np, a.np);
+                                                              local, a.gperm + (size_t)nxt * a.np, a.np, a.err);
             if (threadIdx.x == 0) a.gkey[nxt] = gk;
             __threadfence();
             __syncthreads();
@@ -486,6 +487,7 @@ DpArgs make_args(const Instance& I, const DpsoLaunch& p, void* ws) {
     a.gkey = reinterpret_cast<unsigned long long*>(b + w.gkey);
     a.gperm = reinterpret_cast<int16_t*>(b + w.gperm);
     a.counter = reinterpret_cast<unsigned int*>(b + w.counter);
+    a.err = I.err;
     if (p.peer && I.peer && I.peer->open) {
         a.pw = I.peer->world;
         a.pr = I.peer->rank;

@@ -35,11 +35,21 @@ __device__ __forceinline__ unsigned long long peer_ld_acquire64(const unsigned l
 
 // Whole CTA; `seq` (len entries, global memory) holds this rank's best sequence on entry and the
 // global best's on exit.  Returns the global key (every thread).
+// A rank that never arrives (its process died) must not hang the others: after kPeerTimeoutNs
+// the wait gives up, raises bit 2 of the instance's error flag (cdd_check reports it) and the run
+// continues with an unreliable swarm best.
+constexpr unsigned long long kPeerTimeoutNs = 30ull * 1000 * 1000 * 1000;
+__device__ __forceinline__ unsigned long long peer_globaltimer() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+
 __device__ __forceinline__ unsigned long long peer_exchange_block(uint8_t* const* regions, int world,
                                                                   int rank, int64_t per_rank, int np,
                                                                   uint32_t e, int par,
                                                                   unsigned long long local_key,
-                                                                  int16_t* seq, int len) {
+                                                                  int16_t* seq, int len, int* err) {
     __shared__ unsigned long long s_gk;
     uint8_t* root = regions[0];
     unsigned long long* rkey = reinterpret_cast<unsigned long long*>(root + kPeerKeyOff);
@@ -57,7 +67,14 @@ __device__ __forceinline__ unsigned long long peer_exchange_block(uint8_t* const
         __threadfence_system();
         atomicAdd_system(rarr, 1u);
         const unsigned int target = (unsigned int)world * (e + 1u);
-        while ((int)(peer_ld_acquire(rarr) - target) < 0) __nanosleep(64);
+        const unsigned long long t0 = peer_globaltimer();
+        while ((int)(peer_ld_acquire(rarr) - target) < 0) {
+            __nanosleep(64);
+            if (peer_globaltimer() - t0 > kPeerTimeoutNs) {
+                atomicOr(err, 2);
+                break;
+            }
+        }
         s_gk = peer_ld_acquire64(&rkey[e % 3]);
     }
     __syncthreads();
