@@ -68,7 +68,8 @@ __device__ __forceinline__ unsigned long long peer_exchange_block(uint8_t* const
         atomicAdd_system(rarr, 1u);
         const unsigned int target = (unsigned int)world * (e + 1u);
         const unsigned long long t0 = peer_globaltimer();
-        while ((int)(peer_ld_acquire(rarr) - target) < 0) {
+        // after one timeout the exchange is broken for the rest of the run: no more waiting
+        while (!(*(volatile int*)err & 2) && (int)(peer_ld_acquire(rarr) - target) < 0) {
             __nanosleep(64);
             if (peer_globaltimer() - t0 > kPeerTimeoutNs) {
                 atomicOr(err, 2);
