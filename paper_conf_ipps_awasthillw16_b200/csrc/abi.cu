@@ -707,16 +707,17 @@ int dpso_peer_open(cdd_instance* I, const uint8_t* handles) {
     return CDD_OK;
 }
 
-__global__ void peer_reset_kernel(uint8_t* region) {
+__global__ void peer_reset_kernel(uint8_t* region, int* err) {
     if (threadIdx.x < 3) reinterpret_cast<unsigned long long*>(region + cdd::kPeerKeyOff)[threadIdx.x] = ULLONG_MAX;
     if (threadIdx.x == 3) *reinterpret_cast<unsigned int*>(region + cdd::kPeerArriveOff) = 0u;
+    if (threadIdx.x == 4) atomicAnd(err, ~2);  // a previous run's exchange timeout
 }
 
 int dpso_peer_reset(cdd_instance* I, void* stream) {
     if (!I) return fail(CDD_EINVAL, "instance is NULL");
     if (!I->peer) return fail(CDD_ESTATE, "no peer exchange (dpso_peer_create first)");
     DeviceGuard g(I->device);
-    peer_reset_kernel<<<1, 32, 0, as_stream(stream)>>>(I->peer->region);
+    peer_reset_kernel<<<1, 32, 0, as_stream(stream)>>>(I->peer->region, I->err);
     const cudaError_t e = cudaGetLastError();
     return e == cudaSuccess ? CDD_OK : cuda_fail(e, "dpso_peer_reset");
 }
