@@ -89,3 +89,27 @@ def test_invalid_initial_ids_flagged(lib, lanes):
         lib.cdd_check(ins)
     assert e.value.code == lib.CDD_EDATA
     lib.cdd_check(ins)  # cleared
+
+
+def test_given_sequences_under_the_balanced_schedule(lib):
+    # caller-given initial sequences and a chain offset with more chains than resident slots and a
+    # mostly empty last round: split chains start from their own rows and are resumed from the
+    # handover -- every chain's best equals the oracle's replay
+    import torch
+
+    n, chains, steps, offset = 120, 15000, 37, 777
+    inst = gen.cdd_instance(n, 6, 0.6)
+    ins = lib.Instance.from_gen(inst)
+    init = gen.random_perms(chains, n, 21, ld=n + 8)
+    res = lib.sa_run(ins, chains, steps, seed=41, T0=1800.0, chain_offset=offset, lanes=8,
+                     chain_best=True, init=torch.from_numpy(init).cuda())
+    torch.cuda.synchronize()
+    lib.cdd_check(ins)
+    cb = res["chain_best"].cpu().numpy()
+    pr = oracle.Problem.from_instance(inst)
+    p = oracle.sa_params(chains=chains, steps=steps, seed=41, chain_offset=offset, init=init[:, :n])
+    for c in range(chains):
+        assert oracle.sa_chain(pr, p, 1800.0, offset + c)["E_best"] == cb[c], c
+    pen, perm, gid = lib.best_get(ins)
+    assert pen == cb.min() and gid == offset + int(np.argmin(cb))
+    assert oracle.cdd_eval(pr, perm) == pen
