@@ -21,7 +21,7 @@ _lock = threading.Lock()
 _lib = None
 
 CDD, UCDDCP = 0, 1
-MOVE_PERT_FY, MOVE_SWAP = 0, 1
+MOVE_PERT_FY, MOVE_SWAP, MOVE_INSERT, MOVE_WINDOW = 0, 1, 2, 3
 TAG_SA_INIT, TAG_SA, TAG_T0, TAG_DPSO_INIT, TAG_DPSO = 0x11, 0x12, 0x13, 0x21, 0x22
 WALK_MAX = 64
 
@@ -79,6 +79,7 @@ def _load():
             "or_ucddcp_eval": (i64, [vp, vp, vp, vp]),
             "or_eval_batch": (None, [vp, C.c_int, vp, i64, i64, vp]),
             "or_sa_move": (i32, [i32, i32, i32, u64, u64, u64, vp, vp, vp]),
+            "or_sa_neighbour": (None, [i32, i32, i32, vp, vp, vp, vp]),
             "or_t0": (dbl, [vp, i32, u64, i64]),
             "or_sa_chain": (i64, [vp, vp, dbl, u64, vp, vp, vp, vp]),
             "or_sa_run": (None, [vp, vp, dbl, vp, vp, vp, vp]),
@@ -208,6 +209,19 @@ def sa_move(n, pert, move, seed, g, k):
     u = C.c_double()
     P = _load().or_sa_move(n, pert, move, seed, g, k, _ptr(q), _ptr(s), C.byref(u))
     return q[:P].copy(), s[:P].copy(), u.value
+
+
+def sa_neighbour(s, move, q, sigma):
+    """Alg. 1 line 5: the neighbour of sequence s for the move (q, sigma) drawn by sa_move."""
+    s = np.ascontiguousarray(s, dtype=np.int16)
+    P = len(q)
+    qq = np.zeros(4, dtype=np.int32)
+    ss = np.zeros(4, dtype=np.int32)
+    qq[:P] = q
+    ss[:P] = sigma
+    out = np.zeros_like(s)
+    _load().or_sa_neighbour(len(s), move, P, _ptr(qq), _ptr(ss), _ptr(s), _ptr(out))
+    return out
 
 
 def t0(prob: Problem, problem: int, seed: int, samples: int = 5000) -> float:

@@ -14,7 +14,9 @@
  *                                    shift brute force, n! brute force, V-shape, Theorem 1
  *   or_ucddcp_eval          pinned: Table I worked example (penalty 77), integer-LP brute force,
  *                                    Properties 1-2
- *   or_perm_fy / neighbour  pinned: uniformity (chi-square) on tiny n, FY definition [14]
+ *   or_perm_fy / neighbour  pinned: uniformity (chi-square) on tiny n, FY definition [14];
+ *                           insert: permutation + one-segment rotation + uniform (from, to);
+ *                           window: contiguous positions, uniform start, uniform slot shuffle
  *   or_t0                   pinned: vs numpy population std of independently evaluated samples
  *   or_sa_chain / run       pinned: invariants (greedy at T0=0, best==eval(best perm), n=10 reaches the
  *                                    10! optimum); trajectory "parity unpinned" vs the paper
@@ -79,7 +81,11 @@ void    or_eval_batch(const or_instance *I, int problem, const int16_t *perms, i
                       int64_t batch, int64_t *out);
 
 /* ---- Simulated annealing (Alg. 1; asynchronous chains P:172-179) -------------- */
-enum { OR_MOVE_PERT_FY = 0, OR_MOVE_SWAP = 1 };
+/* Neighbour moves (R11, R11b, R11c): PERT_FY = Pert distinct random positions shuffled by
+ * Fisher-Yates; SWAP = two random positions exchanged; INSERT = the job at a random position
+ * `from` re-inserted at a random position `to` (BASELINE north_star "swap/insertion move");
+ * WINDOW = a contiguous sub-sequence of Pert positions shuffled by Fisher-Yates. */
+enum { OR_MOVE_PERT_FY = 0, OR_MOVE_SWAP = 1, OR_MOVE_INSERT = 2, OR_MOVE_WINDOW = 3 };
 typedef struct {
     int32_t  problem;       /* OR_CDD / OR_UCDDCP                         */
     int64_t  chains;
@@ -97,9 +103,13 @@ typedef struct {
 } or_sa_params;
 
 /* The neighbour move of SA step k of chain g: Pert distinct positions q[0..P-1] (ascending),
- * sigma = FY permutation of the P slots (slot i receives the old job of slot sigma[i]), u = rand(0,1). */
+ * sigma = FY permutation of the P slots (slot i receives the old job of slot sigma[i]), u = rand(0,1).
+ * INSERT: q = (from, to) in draw order, sigma = identity.  WINDOW: q consecutive. */
 int32_t or_sa_move(int32_t n, int32_t pert, int32_t move, uint64_t seed, uint64_t g, uint64_t k,
                    int32_t q[4], int32_t sigma[4], double *u);
+/* Alg. 1 line 5: s_new = Neighbour(s) for the move drawn by or_sa_move. */
+void or_sa_neighbour(int32_t n, int32_t move, int32_t P, const int32_t q[4], const int32_t sigma[4],
+                     const int16_t *s, int16_t *s_new);
 /* T0 = population standard deviation of the fitness of `samples` random sequences. */
 double  or_t0(const or_instance *I, int32_t problem, uint64_t seed, int64_t samples);
 /* One chain. Returns E_best; best_J (n) = best sequence; final_E/final_J optional; trace optional:

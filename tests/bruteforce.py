@@ -107,3 +107,32 @@ def v_shaped(P, a, b, J) -> bool:
 
 def all_sequences(n):
     return [list(p) for p in itertools.permutations(range(n))]
+
+
+def breakpoint_bf(P, a, b, d, J, X=None, g=None):
+    """Exact (Python integers, any magnitude) min over integer starts s >= 0 of the no-idle
+    objective eq. (1)/(2).  The objective is convex piecewise linear in s with breakpoints where
+    some job completes exactly at d, so the minimum over s in [0, inf) is attained at s = 0 or at
+    one of the starts s = d - C_k >= 0 (C_k = completion time of position k when starting at 0)."""
+    d = int(d)
+    C, cands = 0, {0}
+    for k, j in enumerate(J):
+        C += int(P[j]) - (0 if X is None else int(X[k]))
+        if d - C >= 0:
+            cands.add(d - C)
+    return min(objective(P, a, b, d, J, s, X, g) for s in cands)
+
+
+def ucddcp_vertex_bf(P, a, b, d, J, M, g):
+    """Exact UCDDCP for a fixed sequence with d >= sum P: every compression vector with X_k in
+    {0, P_k - M_k} (the LP's vertices in X: for a fixed start the objective is linear in each X_k
+    between two breakpoints, so an optimum exists at an extreme compression -- checked against the
+    integer DP on small values) times the exact start enumeration."""
+    n = len(J)
+    full = [int(P[j]) - int(M[j]) for j in J]
+    best = None
+    for mask in range(1 << n):
+        X = [full[k] if (mask >> k) & 1 else 0 for k in range(n)]
+        z = breakpoint_bf(P, a, b, d, J, X, g)
+        best = z if best is None or z < best else best
+    return best

@@ -215,3 +215,51 @@ def test_eval_batch_matches_single():
     assert list(out) == [oracle.cdd_eval(pr, r[:50]) for r in perms]
     outt = oracle.eval_batch_threaded(pr, perms, threads=3)
     assert list(outt) == list(out)
+
+
+# ------------------------------------------------- wide value ranges (the generic path, §8(b))
+def _wide_cases(count, nmax, seed, pmax, wmax, rng_h=True):
+    rng = np.random.default_rng(seed)
+    for c in range(count):
+        n = int(rng.integers(1, nmax + 1))
+        P = rng.integers(1, pmax + 1, n).astype(np.int64)
+        a = rng.integers(0, wmax + 1, n).astype(np.int64)
+        b = rng.integers(0, wmax + 1, n).astype(np.int64)
+        M = (P - rng.integers(0, P)).astype(np.int64)           # 1 <= M <= P
+        g = rng.integers(0, wmax + 1, n).astype(np.int64)
+        h = float(rng.choice([0.0, 0.2, 0.4, 0.6, 0.8, 1.0, 1.3])) if rng_h else 1.0
+        d = int(h * int(P.sum()))
+        yield P, a, b, M, g, d, rng.permutation(n)
+
+
+def test_cdd_wide_values_vs_breakpoint_bruteforce():
+    # P:29-59 define P, alpha, beta, d as general non-negative integers: p <= 1000,
+    # alpha, beta <= 10^4, and n up to 300 (exact big-integer brute force over starts)
+    for P, a, b, M, g, d, J in _wide_cases(300, 12, 21, 1000, 10_000):
+        pr = oracle.Problem(P, a, b, d)
+        assert oracle.cdd_eval(pr, J) == bf.breakpoint_bf(P, a, b, d, J)
+    for P, a, b, M, g, d, J in _wide_cases(12, 300, 22, 1000, 10_000):
+        pr = oracle.Problem(P, a, b, d)
+        assert oracle.cdd_eval(pr, J) == bf.breakpoint_bf(P, a, b, d, J)
+
+
+def test_cdd_huge_values_int64_exact():
+    # penalties far beyond 2^32: int32 data at the top of its range, exact in int64
+    for P, a, b, M, g, d, J in _wide_cases(60, 9, 23, 2_000_000, 200_000_000):
+        pr = oracle.Problem(P, a, b, d)
+        z = bf.breakpoint_bf(P, a, b, d, J)
+        assert z < 2**63 and oracle.cdd_eval(pr, J) == z
+    # shift brute force on moderate values agrees with the breakpoint enumeration (pins the helper)
+    for P, a, b, M, g, d, J in _wide_cases(100, 6, 24, 30, 50):
+        assert bf.breakpoint_bf(P, a, b, d, J) == bf.shift_bf(P, a, b, d, J)
+
+
+def test_ucddcp_wide_values_vs_vertex_bruteforce():
+    for P, a, b, M, g, d, J in _wide_cases(150, 8, 25, 1000, 10_000, rng_h=False):
+        d = int(P.sum()) + int(P[0])
+        pr = oracle.Problem(P, a, b, d, M, g)
+        assert oracle.ucddcp_eval(pr, J) == bf.ucddcp_vertex_bf(P, a, b, d, J, M, g)
+    # the vertex enumeration equals the integer DP (no Property 2 assumed) on small values
+    for P, a, b, M, g, d, J in _wide_cases(60, 5, 26, 6, 6, rng_h=False):
+        d = int(P.sum())
+        assert bf.ucddcp_vertex_bf(P, a, b, d, J, M, g) == bf.dp_schedule(P, a, b, d, J, M=M, g=g)

@@ -317,3 +317,91 @@ def test_dpso_n10_reaches_optimum():
     z_opt = int(oracle.eval_batch_threaded(pr, gen.all_perms(10)).min())
     r = oracle.dpso_run(pr, oracle.dpso_params(particles=128, iters=200, seed=5))
     assert r["E_best"] == z_opt
+
+
+# ------------------------------------------------------------ insertion and window moves
+def test_insert_move_is_uniform_ordered_pair():
+    # BASELINE north_star "swap/insertion move" (R11b): (from, to) are two distinct positions in
+    # the order of the two Floyd draws -- every ordered pair of distinct positions equally likely
+    n, N = 5, 40000
+    counts = {}
+    for k in range(N):
+        q, s, u = oracle.sa_move(n, 4, oracle.MOVE_INSERT, 23, 1, k)
+        assert len(q) == 2 and q[0] != q[1] and 0 <= q.min() and q.max() < n and 0.0 < u < 1.0
+        counts[tuple(q)] = counts.get(tuple(q), 0) + 1
+    assert len(counts) == n * (n - 1)
+    e = N / (n * (n - 1))
+    assert sum((c - e) ** 2 / e for c in counts.values()) < 60  # 19 dof
+
+
+def test_insert_neighbour_definition():
+    # insertion: the moved job lands at `to`, and deleting it from both sequences leaves the same
+    # sequence (every other job keeps its relative order) -- checked against that definition
+    rng = np.random.default_rng(7)
+    for t in range(400):
+        n = int(rng.integers(2, 40))
+        s = rng.permutation(n).astype(np.int16)
+        k = int(rng.integers(0, 1 << 30))
+        q, sig, _ = oracle.sa_move(n, 4, oracle.MOVE_INSERT, 3, 9, k)
+        f, to = int(q[0]), int(q[1])
+        s2 = oracle.sa_neighbour(s, oracle.MOVE_INSERT, q, sig)
+        assert sorted(s2.tolist()) == list(range(n))
+        assert s2[to] == s[f]
+        assert [x for x in s2.tolist() if x != s[f]] == [x for x in s.tolist() if x != s[f]]
+        lo, hi = min(f, to), max(f, to)
+        assert np.array_equal(s2[:lo], s[:lo]) and np.array_equal(s2[hi + 1:], s[hi + 1:])
+
+
+def test_window_move_contiguous_uniform():
+    # "A sub-sequence of size Pert=4 is selected ... Fisher Yates ... on this sub-sequence
+    # while retaining the position of other jobs" (R11c)
+    n, N = 9, 30000
+    starts, sigmas = {}, {}
+    rng = np.random.default_rng(1)
+    for k in range(N):
+        q, sig, u = oracle.sa_move(n, 4, oracle.MOVE_WINDOW, 31, 4, k)
+        assert list(q) == list(range(q[0], q[0] + 4)) and q[-1] < n
+        assert sorted(sig) == [0, 1, 2, 3]
+        starts[int(q[0])] = starts.get(int(q[0]), 0) + 1
+        sigmas[tuple(sig)] = sigmas.get(tuple(sig), 0) + 1
+        if k < 300:
+            s = rng.permutation(n).astype(np.int16)
+            s2 = oracle.sa_neighbour(s, oracle.MOVE_WINDOW, q, sig)
+            out = np.ones(n, bool)
+            out[q] = False
+            assert np.array_equal(s2[out], s[out]) and sorted(s2[q]) == sorted(s[q])
+    assert len(starts) == n - 3 and len(sigmas) == 24
+    e1, e2 = N / (n - 3), N / 24
+    assert sum((c - e1) ** 2 / e1 for c in starts.values()) < 30   # 5 dof
+    assert sum((c - e2) ** 2 / e2 for c in sigmas.values()) < 70   # 23 dof
+    # Pert-FY and window share the slot shuffle words (same sigma for the same step)
+    for k in range(50):
+        assert list(oracle.sa_move(n, 4, oracle.MOVE_WINDOW, 31, 4, k)[1]) == \
+            list(oracle.sa_move(n, 4, oracle.MOVE_PERT_FY, 31, 4, k)[1])
+
+
+@pytest.mark.parametrize("move", [oracle.MOVE_INSERT, oracle.MOVE_WINDOW])
+def test_sa_chain_with_other_moves_is_alg1(move):
+    inst, pr, p = _sa(n=35, steps=500, seed=13, move=move)
+    T0 = oracle.t0(pr, oracle.CDD, 13, 400)
+    r = oracle.sa_chain(pr, p, T0, 3, trace=True)
+    assert oracle.cdd_eval(pr, r["best"]) == r["E_best"]
+    # replay with the oracle's own move + neighbour: every E_new is the penalty of the neighbour
+    s = oracle.perm_fy(inst.n, 13, oracle.TAG_SA_INIT, 3)
+    for k, (En, acc) in enumerate(zip(r["E_new"], r["accepted"])):
+        q, sig, _ = oracle.sa_move(inst.n, 4, move, 13, 3, k)
+        s_new = oracle.sa_neighbour(s, move, q, sig)
+        assert oracle.cdd_eval(pr, s_new) == En
+        if acc:
+            s = s_new
+    assert np.array_equal(s, r["final"])
+
+
+@pytest.mark.parametrize("move", [oracle.MOVE_INSERT, oracle.MOVE_WINDOW])
+def test_sa_other_moves_reach_n10_optimum(move):
+    inst = gen.cdd_instance(10, 1, 0.4)
+    pr = oracle.Problem.from_instance(inst)
+    z_opt = int(oracle.eval_batch_threaded(pr, gen.all_perms(10)).min())
+    p = oracle.sa_params(chains=64, steps=1000, seed=0x5EED0001, move=move)
+    r = oracle.sa_run(pr, p, oracle.t0(pr, oracle.CDD, 0x5EED0001))
+    assert r["E_best"] == z_opt
