@@ -50,9 +50,16 @@ typedef enum {
 
 typedef enum { CDD_PROBLEM_CDD = 0, CDD_PROBLEM_UCDDCP = 1 } cdd_problem;
 
-/* SA neighbourhood: the paper's move (Pert jobs at random positions shuffled by Fisher-Yates,
- * P:192) or a plain swap of two random positions. */
-typedef enum { CDD_MOVE_PERT_FY = 0, CDD_MOVE_SWAP = 1 } cdd_move;
+/* SA neighbourhood (readings R11, R11b, R11c):
+ *   CDD_MOVE_PERT_FY  the paper's move: Pert jobs at random positions (Floyd sample)
+ *                     shuffled by Fisher-Yates over their slots;
+ *   CDD_MOVE_SWAP     two random positions exchanged;
+ *   CDD_MOVE_INSERT   the job at a random position `from` is re-inserted at a random position
+ *                     `to` != from, the jobs in between move one place towards `from`
+ *                     ((from, to) uniform over ordered pairs; BASELINE "swap/insertion move");
+ *   CDD_MOVE_WINDOW   the contiguous sub-sequence of Pert positions at a random start shuffled by
+ *                     Fisher-Yates ("A sub-sequence of size Pert=4 is selected"). */
+typedef enum { CDD_MOVE_PERT_FY = 0, CDD_MOVE_SWAP = 1, CDD_MOVE_INSERT = 2, CDD_MOVE_WINDOW = 3 } cdd_move;
 
 typedef struct cdd_instance cdd_instance; /* opaque, library-owned, bound to one device */
 
@@ -261,14 +268,16 @@ CDD_API int dpso_end(cdd_instance *inst, const dpso_params *params, void *worksp
  *   dpso_peer_open(handles [world * CDD_IPC_HANDLE_BYTES]): maps every other rank's region;
  *   dpso_peer_reset(stream): re-arms this rank's region -- before EVERY run, followed by a
  *       cross-process barrier after the stream has completed (no rank may start before rank 0's
- *       region is re-armed);
+ *       region is re-armed); a fused run without a reset since the previous one returns
+ *       CDD_ESTATE;
  *   dpso_run_peer(params): the whole run (as dpso_run) with particle_offset = rank * particles
  *       (equal shares); every rank must call it (the kernels wait for each other: all ranks'
  *       kernels must be able to run concurrently -- one GPU per rank, or time-sliced processes);
  *   dpso_peer_destroy: unmaps and frees (also done by cdd_instance_destroy).
  * Results are identical to one GPU running all particles (same Philox streams, same ties).
  * A rank that never arrives at an exchange (its process died) does not hang the others: after 30 s
- * the wait gives up and cdd_check reports CDD_EDATA ("a peer rank never reached ...").
+ * the wait gives up, cdd_check reports CDD_EDATA ("a peer rank never reached ..."), and from then
+ * on every rank continues with its own device-local swarm best (no peer memory is read).
  * CDD_ESTATE on a wrong order of calls; CDD_ECUDA if IPC is unavailable. */
 #define CDD_IPC_HANDLE_BYTES 64
 CDD_API int dpso_peer_create(cdd_instance *inst, int world, int rank, uint8_t *ipc_handle);

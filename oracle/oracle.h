@@ -125,8 +125,8 @@ void    or_sa_run(const or_instance *I, const or_sa_params *p, double T0, int64_
  * runs a Markov chain of p->steps (= M) moves at the constant temperature T_j (T_0 = T0,
  * T_{j+1} = T_j * mu); move m of level j uses the counters of step k = j*M + m.  The final state of
  * minimal cost over all chains (ties: lowest global id) is s^min_j, the initial state of every chain
- * at level j+1.  Outputs: best-ever penalty / chain / level / sequence (within a level min over
- * chains of (E_best, g); a later level replaces it only if strictly better), level_min_E[j] =
+ * at level j+1.  Outputs: best-ever penalty / chain / level / sequence (the minimum of (E_best, g)
+ * over all levels and chains; an exact tie keeps the earlier level), level_min_E[j] =
  * E(s^min_j) and level_min_g[j] (either may be NULL). */
 void or_sa_sync(const or_instance *I, const or_sa_params *p, double T0, int64_t levels,
                 int64_t *best_E, uint64_t *best_g, int64_t *best_level, int16_t *best_J,

@@ -28,7 +28,7 @@ _lib = C.CDLL(_SO)
 
 CDD_OK, CDD_EINVAL, CDD_ERANGE, CDD_ENOMEM, CDD_ECUDA, CDD_ESTATE, CDD_EDATA = 0, -1, -2, -3, -4, -5, -6
 PROBLEMS = {"cdd": 0, "ucddcp": 1}
-MOVES = {"pert_fy": 0, "swap": 1}
+MOVES = {"pert_fy": 0, "swap": 1, "insert": 2, "window": 3}
 
 
 class CddError(RuntimeError):

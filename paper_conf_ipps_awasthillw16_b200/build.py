@@ -10,7 +10,9 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 OUT = os.path.join(HERE, "libcdd.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
-SOURCES = ["abi.cu", "eval.cu", "eval2.cu", "sa.cu", "dpso.cu", "schedule.cu"]
+SOURCES = ["abi.cu", "eval.cu", "eval2.cu", "sa.cu", "dpso.cu", "schedule.cu", "sag_cdd.cu",
+           "sag_cdd_tr.cu", "sag_ucd.cu", "sag_ucd_tr.cu", "sag_cdd_ins.cu", "sag_cdd_ins_tr.cu",
+           "sag_ucd_ins.cu", "sag_ucd_ins_tr.cu"]
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
          "-Xcompiler", "-fPIC", "-Xcompiler", "-fvisibility=hidden", "--expt-relaxed-constexpr",
          "-Xptxas", "-v"]
@@ -36,7 +38,7 @@ def build(force: bool = False, verbose: bool = False, out: str = OUT, extra=()) 
             raise RuntimeError(f"nvcc failed for {src}:\n{r.stderr}")
         return obj, r.stderr
 
-    with cf.ThreadPoolExecutor(max_workers=len(SOURCES)) as ex:
+    with cf.ThreadPoolExecutor(max_workers=min(len(SOURCES), os.cpu_count() or 4)) as ex:
         results = list(ex.map(compile_one, SOURCES))
     if verbose:
         for _, log in results:

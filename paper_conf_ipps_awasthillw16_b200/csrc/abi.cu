@@ -374,7 +374,9 @@ static int sa_validate(const cdd_instance* I, const sa_params* p, cdd::SaLaunch*
     if (p->steps < 0 || p->steps >= (int64_t)UINT32_MAX) return fail(CDD_EINVAL, "steps must be in [0, 2^32)");
     if (p->chain_offset + (uint64_t)p->chains > (1ull << 32)) return fail(CDD_EINVAL, "chain ids must fit 32 bits");
     if (p->pert < 1 || p->pert > 4) return fail(CDD_EINVAL, "pert must be in [1, 4]");
-    if (p->move != CDD_MOVE_PERT_FY && p->move != CDD_MOVE_SWAP) return fail(CDD_EINVAL, "bad move");
+    if (p->move != CDD_MOVE_PERT_FY && p->move != CDD_MOVE_SWAP && p->move != CDD_MOVE_INSERT &&
+        p->move != CDD_MOVE_WINDOW)
+        return fail(CDD_EINVAL, "bad move");
     if (!std::isfinite(p->mu) || p->mu < 0) return fail(CDD_EINVAL, "mu must be finite and >= 0");
     if (!(p->T0 > 0) && !p->T0_in && p->t0_samples < 1) return fail(CDD_EINVAL, "T0 <= 0 needs t0_samples >= 1");
     if (std::isnan(p->T0)) return fail(CDD_EINVAL, "T0 is NaN");
@@ -464,8 +466,9 @@ int sa_sync_run_peer(cdd_instance* I, const sa_sync_params* q, void* ws, size_t 
     cdd::SaLaunch L{};
     const int rc = sync_validate(I, q, &L);
     if (rc != CDD_OK) return rc;
-    const cdd::DpsoPeer* P = I->peer;
+    cdd::DpsoPeer* P = I->peer;
     if (!P || !P->open) return fail(CDD_ESTATE, "peer exchange not open (dpso_peer_create / dpso_peer_open)");
+    if (!P->armed) return fail(CDD_ESTATE, "peer exchange not re-armed: dpso_peer_reset (+ a barrier) before every fused run");
     if (q->chain_offset != (uint64_t)P->rank * (uint64_t)q->chains)
         return fail(CDD_EINVAL, "chain_offset must be rank * chains (equal shares)");
     DeviceGuard g(I->device);
@@ -473,6 +476,7 @@ int sa_sync_run_peer(cdd_instance* I, const sa_sync_params* q, void* ws, size_t 
     if (!ws || ws_bytes < need)
         return fail(CDD_ENOMEM, "workspace too small: need " + std::to_string(need) + " bytes");
     L.peer = true;
+    P->armed = false;
     for (int64_t j = 0; j < q->levels; ++j) {
         const cudaError_t e = cdd::launch_sa_sync_level(*I, L, j, q->level_min, ws, as_stream(stream));
         if (e != cudaSuccess) return cuda_fail(e, "sa_sync_run_peer");
@@ -719,7 +723,9 @@ int dpso_peer_reset(cdd_instance* I, void* stream) {
     DeviceGuard g(I->device);
     peer_reset_kernel<<<1, 32, 0, as_stream(stream)>>>(I->peer->region, I->err);
     const cudaError_t e = cudaGetLastError();
-    return e == cudaSuccess ? CDD_OK : cuda_fail(e, "dpso_peer_reset");
+    if (e != cudaSuccess) return cuda_fail(e, "dpso_peer_reset");
+    I->peer->armed = true;
+    return CDD_OK;
 }
 
 int dpso_peer_destroy(cdd_instance* I) {
@@ -740,13 +746,15 @@ int dpso_run_peer(cdd_instance* I, const dpso_params* p, void* ws, size_t ws_byt
     cdd::DpsoLaunch L{};
     int rc = dpso_prepare(I, p, ws, ws_bytes, &L);
     if (rc != CDD_OK) return rc;
-    const cdd::DpsoPeer* P = I->peer;
+    cdd::DpsoPeer* P = I->peer;
     if (!P || !P->open) return fail(CDD_ESTATE, "peer exchange not open (dpso_peer_create / dpso_peer_open)");
+    if (!P->armed) return fail(CDD_ESTATE, "peer exchange not re-armed: dpso_peer_reset (+ a barrier) before every fused run");
     if (p->particle_offset != (uint64_t)P->rank * (uint64_t)p->particles)
         return fail(CDD_EINVAL, "particle_offset must be rank * particles (equal shares)");
     if ((uint64_t)p->particles * (uint64_t)P->world > (1ull << 32))
         return fail(CDD_EINVAL, "global particle ids must fit 32 bits");
     L.peer = true;
+    P->armed = false;
     DeviceGuard g(I->device);
     cudaStream_t s = as_stream(stream);
     cudaError_t e = cdd::dpso_begin(*I, L, ws, s);

@@ -32,6 +32,7 @@ struct DpsoPeer {
     std::vector<uint8_t*> mapped;    // peers' regions opened in this process (own slot: nullptr)
     uint8_t** d_regions = nullptr;   // device [world]: region of every rank (own included)
     bool open = false;
+    bool armed = false;  // dpso_peer_reset since the last fused run (host-side call-order check)
 };
 
 struct Instance {
@@ -136,5 +137,35 @@ void dpso_gbest(const Instance& I, const DpsoLaunch& p, void* ws, int64_t t, int
 cudaError_t dpso_end(Instance& I, const DpsoLaunch& p, void* ws, cudaStream_t s);
 
 int sa_e_for_n(int n);  // elements per lane of the warp-per-chain kernels
+
+// ---- group-kernel SA variants (sag_*.cu: one translation unit per problem / trace / move class)
+struct GroupCfg {
+    int G, E;  // G = 0: warp-per-chain kernel
+};
+#define CDD_SAG_DECL(NAME)                                                                      \
+    size_t NAME##_ws(const Instance& I, const SaLaunch& p, GroupCfg cfg);                      \
+    cudaError_t NAME##_run(Instance& I, const SaLaunch& p, GroupCfg cfg, void* ws, cudaStream_t s);
+#define CDD_SAG_SYNC_DECL(NAME)                                                                 \
+    size_t NAME##_sync_ws(const Instance& I, const SaLaunch& p, GroupCfg cfg);                 \
+    cudaError_t NAME##_sync_level(Instance& I, const SaLaunch& p, GroupCfg cfg, int64_t j,     \
+                                  int64_t* level_min, void* ws, cudaStream_t s);               \
+    void NAME##_sync_ptrs(const Instance& I, const SaLaunch& p, GroupCfg cfg, void* ws,        \
+                          unsigned long long** key, int16_t** perm);
+CDD_SAG_DECL(sag_cdd)
+CDD_SAG_DECL(sag_cdd_tr)
+CDD_SAG_DECL(sag_ucd)
+CDD_SAG_DECL(sag_ucd_tr)
+CDD_SAG_DECL(sag_cdd_ins)
+CDD_SAG_DECL(sag_cdd_ins_tr)
+CDD_SAG_DECL(sag_ucd_ins)
+CDD_SAG_DECL(sag_ucd_ins_tr)
+CDD_SAG_SYNC_DECL(sag_cdd)
+CDD_SAG_SYNC_DECL(sag_ucd)
+CDD_SAG_SYNC_DECL(sag_cdd_ins)
+CDD_SAG_SYNC_DECL(sag_ucd_ins)
+cudaError_t sag_cdd_t0(const Instance& I, GroupCfg cfg, uint64_t seed, int64_t samples, double* T0_dev,
+                       void* ws, cudaStream_t s);
+cudaError_t sag_ucd_t0(const Instance& I, GroupCfg cfg, uint64_t seed, int64_t samples, double* T0_dev,
+                       void* ws, cudaStream_t s);
 
 }  // namespace cdd

@@ -36,8 +36,9 @@ __device__ __forceinline__ unsigned long long peer_ld_acquire64(const unsigned l
 // Whole CTA; `seq` (len entries, global memory) holds this rank's best sequence on entry and the
 // global best's on exit.  Returns the global key (every thread).
 // A rank that never arrives (its process died) must not hang the others: after kPeerTimeoutNs
-// the wait gives up, raises bit 2 of the instance's error flag (cdd_check reports it) and the run
-// continues with an unreliable swarm best.
+// the wait gives up, raises bit 2 of the instance's error flag (cdd_check reports it), and this
+// and every later exchange of the run keep the LOCAL key and sequence (no peer memory is read
+// once the exchange is broken: the winner could be the dead rank, or its slot already re-armed).
 constexpr unsigned long long kPeerTimeoutNs = 30ull * 1000 * 1000 * 1000;
 __device__ __forceinline__ unsigned long long peer_globaltimer() {
     unsigned long long t;
@@ -51,6 +52,7 @@ __device__ __forceinline__ unsigned long long peer_exchange_block(uint8_t* const
                                                                   unsigned long long local_key,
                                                                   int16_t* seq, int len, int* err) {
     __shared__ unsigned long long s_gk;
+    __shared__ int s_owner;
     uint8_t* root = regions[0];
     unsigned long long* rkey = reinterpret_cast<unsigned long long*>(root + kPeerKeyOff);
     unsigned int* rarr = reinterpret_cast<unsigned int*>(root + kPeerArriveOff);
@@ -76,11 +78,18 @@ __device__ __forceinline__ unsigned long long peer_exchange_block(uint8_t* const
                 break;
             }
         }
-        s_gk = peer_ld_acquire64(&rkey[e % 3]);
+        unsigned long long gk = peer_ld_acquire64(&rkey[e % 3]);
+        // validate before any peer read: a broken exchange, an empty key or an owner outside the
+        // world fall back to this rank's own best
+        const unsigned long long own = gk == ULLONG_MAX ? ~0ull : (gk & 0xffffffffull) / (unsigned long long)per_rank;
+        const bool ok = !(*(volatile int*)err & 2) && gk != ULLONG_MAX && own < (unsigned long long)world &&
+                        gk <= local_key;
+        s_gk = ok ? gk : local_key;
+        s_owner = ok ? (int)own : rank;
     }
     __syncthreads();
     const unsigned long long gk = s_gk;
-    const int owner = (int)((gk & 0xffffffffull) / (unsigned long long)per_rank);
+    const int owner = s_owner;
     if (owner != rank) {
         const volatile int16_t* src = reinterpret_cast<const int16_t*>(regions[owner] + kPeerPermOff) + (size_t)par * np;
         for (int i = threadIdx.x; i < len; i += blockDim.x) seq[i] = src[i];

@@ -1,0 +1,8 @@
+// sag_ucd_ins.cu -- group-kernel SA instantiations: UCDDCP, trace off, insertion move
+// (sa_impl.cuh; one translation unit per variant so nvcc compiles them in parallel).
+#include "sa_impl.cuh"
+
+namespace cdd {
+CDD_SAG_VARIANT(sag_ucd_ins, true, false, 1)
+CDD_SAG_SYNC_VARIANT(sag_ucd_ins, true, 1)
+}  // namespace cdd

@@ -1,0 +1,7 @@
+// sag_ucd_ins_tr.cu -- group-kernel SA instantiations: UCDDCP, trace on, insertion move
+// (sa_impl.cuh; one translation unit per variant so nvcc compiles them in parallel).
+#include "sa_impl.cuh"
+
+namespace cdd {
+CDD_SAG_VARIANT(sag_ucd_ins_tr, true, true, 1)
+}  // namespace cdd

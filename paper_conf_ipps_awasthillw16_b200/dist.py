@@ -19,14 +19,43 @@ def owner_rank(key: int, ids_per_rank: int) -> int:
     return int(key & 0xFFFFFFFF) // int(ids_per_rank)
 
 
+# The library's keys are unsigned 64-bit (penalty << 32 | id) with the empty key 0xFFFF...FFFF; the
+# collectives see them as signed int64.  Valid keys are < 2^63 (penalties < 2^31), so only the empty
+# key (-1 when signed) must be lifted to INT64_MAX before a MIN and restored afterwards.
+_EMPTY_SIGNED = -1
+_INT64_MAX = (1 << 63) - 1
+
+
+def _lift_empty(key: torch.Tensor) -> None:
+    key.masked_fill_(key == _EMPTY_SIGNED, _INT64_MAX)
+
+
+def _restore_empty(key: torch.Tensor) -> None:
+    key.masked_fill_(key == _INT64_MAX, _EMPTY_SIGNED)
+
+
 def reduce_best(key: torch.Tensor, perm: torch.Tensor, ids_per_rank: int, group=None) -> int:
-    """In place: key <- MIN over ranks; perm <- the winner's perm.  Returns the winner's rank.
+    """In place: key <- MIN over ranks; perm <- the winner's perm.  Returns the winner's rank
+    (-1 if no rank holds a result; key and perm are then left empty / unchanged).
 
     `key` is an int64 [1] tensor, `perm` an int16 [n] tensor (device tensors with NCCL, CPU tensors
     with gloo).  One all-reduce and one broadcast; the broadcast source is known to every rank
-    from the reduced key, so no extra round trip is needed."""
+    from the reduced key.  Raises if the owner computed from the key is not a rank that holds it
+    (two ranks with overlapping id ranges, or a wrong ids_per_rank)."""
+    local = key.clone()
+    _lift_empty(key)
     dist.all_reduce(key, op=dist.ReduceOp.MIN, group=group)
-    src = owner_rank(int(key.item()), ids_per_rank)
+    k = int(key.item())
+    if k == _INT64_MAX:
+        _restore_empty(key)
+        return -1
+    src = owner_rank(k, ids_per_rank)
+    if not 0 <= src < dist.get_world_size(group):
+        raise RuntimeError(f"best key {k:#x}: owner rank {src} outside the world")
+    hit = torch.tensor([1 if int(local.item()) == k else 0], dtype=torch.int64, device=key.device)
+    dist.all_reduce(hit, op=dist.ReduceOp.SUM, group=group)
+    if int(hit.item()) != 1:
+        raise RuntimeError(f"best key {k:#x} held by {int(hit.item())} ranks (ids must be disjoint)")
     dist.broadcast(perm.view(torch.uint8), src=src, group=group)
     return src
 
@@ -36,10 +65,15 @@ def reduce_best_async(key: torch.Tensor, perm: torch.Tensor, group=None) -> None
     MIN-all-reduced, every rank but the owner (whose local key equals the minimum -- keys are
     unique, they carry the global id) zeroes its sequence, and the sequences are SUM-all-reduced as
     bytes, which leaves exactly the owner's.  Two collectives queued on the stream, so a loop of
-    exchanges (DPSO iterations, synchronous-SA levels) never waits on the host."""
+    exchanges (DPSO iterations, synchronous-SA levels) never waits on the host.  Ranks without a
+    result (empty key) never win; if no rank has one the key stays empty and the sequences sum to
+    zero.  Uniqueness of the winner is the caller's contract (disjoint id ranges); reduce_best
+    checks it."""
     local = key.clone()
+    _lift_empty(key)
     dist.all_reduce(key, op=dist.ReduceOp.MIN, group=group)
-    perm.mul_((local == key).to(perm.dtype))
+    perm.mul_(((local == key) & (key != _INT64_MAX)).to(perm.dtype))
+    _restore_empty(key)
     dist.all_reduce(perm.view(torch.uint8), op=dist.ReduceOp.SUM, group=group)
 
 

@@ -117,3 +117,57 @@ def test_reduce_best_async_equals_broadcast_version():
         k1, k2, p1, p2 = rows[0]
         assert k1 == k2 and p1 == p2
         assert all(r == rows[0] for r in rows)  # every rank holds the same winner
+
+
+def _worker_empty(rank, world, port, q):
+    import sys
+
+    sys.path.insert(0, ROOT)
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    from paper_conf_ipps_awasthillw16_b200.dist import reduce_best, reduce_best_async
+
+    out = []
+    perm = torch.full((11,), rank + 1, dtype=torch.int16)
+    # (a) rank 1 has no result (empty key 0xFFFF...FFFF = -1 signed): rank 0 / 2 must win
+    key = (5 << 32) | (rank * 10) if rank != 1 else -1
+    for fn in (reduce_best, reduce_best_async):
+        k = torch.tensor([key], dtype=torch.int64)
+        p = perm.clone()
+        fn(k, p, 10) if fn is reduce_best else fn(k, p)
+        out.append((int(k.item()), p.tolist()))
+    # (b) nobody has a result: the key stays empty
+    k = torch.tensor([-1], dtype=torch.int64)
+    src = reduce_best(k, perm.clone(), 10)
+    out.append((int(k.item()), src))
+    k = torch.tensor([-1], dtype=torch.int64)
+    reduce_best_async(k, perm.clone())
+    out.append((int(k.item()), None))
+    # (c) two ranks claiming the same key (overlapping ids) is detected
+    k = torch.tensor([(1 << 32) | 3], dtype=torch.int64)
+    try:
+        reduce_best(k, perm.clone(), 10)
+        out.append("no error")
+    except RuntimeError as e:
+        out.append("error")
+    q.put((rank, out))
+    dist.destroy_process_group()
+
+
+def test_reduce_best_empty_keys_and_collisions():
+    # the empty key must never win a signed MIN; a collision must not pass silently
+    world = 3
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    ps = [ctx.Process(target=_worker_empty, args=(r, world, port, q)) for r in range(world)]
+    [p.start() for p in ps]
+    res = dict(q.get(timeout=120) for _ in range(world))
+    [p.join(timeout=60) for p in ps]
+    assert all(p.exitcode == 0 for p in ps)
+    for r in range(world):
+        a, b, c, d, e = res[r]
+        assert a == ((5 << 32) | 0, [1] * 11) and b == a
+        assert c == (-1, -1) and d == (-1, None)
+        assert e == "error"

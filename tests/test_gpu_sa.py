@@ -34,6 +34,9 @@ def test_t0_bit_exact(lib, n, problem):
     assert t_gpu == t_ref  # same double, bit for bit
 
 
+ORACLE_MOVES = {"pert_fy": oracle.MOVE_PERT_FY, "swap": oracle.MOVE_SWAP,
+                "insert": oracle.MOVE_INSERT, "window": oracle.MOVE_WINDOW}
+
 # threads per chain: 32 = warp kernel, 16 / 8 / 4 = group kernel (2 / 4 / 8 chains per warp)
 LANES = [32, 16, 8, 4]
 
@@ -57,8 +60,7 @@ def _run_both(lib, inst, problem, chains, steps, seed, T0=0.0, samples=5000, mov
     T0_ref = T0 if T0 > 0 else oracle.t0(pr, P, seed, samples)
     assert float(res["T0"].item()) == T0_ref
     p = oracle.sa_params(problem=P, chains=chains, steps=steps, mu=mu, pert=pert,
-                         move=oracle.MOVE_SWAP if move == "swap" else oracle.MOVE_PERT_FY,
-                         seed=seed, chain_offset=chain_offset)
+                         move=ORACLE_MOVES[move], seed=seed, chain_offset=chain_offset)
     return ins, res, (pen, perm, gid), pr, p, T0_ref
 
 
@@ -129,6 +131,55 @@ def test_move_variants(lib, move, pert, lanes):
         assert np.array_equal(tr[c] >> 1, ref["E_new"]), c
     full = oracle.sa_run(pr, p, T0)
     assert (pen, gid) == (full["E_best"], full["g"])
+
+
+@pytest.mark.parametrize("lanes", LANES)
+@pytest.mark.parametrize("move", ["insert", "window"])
+@pytest.mark.parametrize("n,problem,chains,steps,mu", [
+    (2, "cdd", 16, 50, 0.88), (9, "cdd", 24, 300, 1.0), (64, "cdd", 40, 400, 1.0),
+    (130, "ucddcp", 24, 300, 1.0), (257, "cdd", 24, 300, 0.995), (1000, "cdd", 12, 200, 1.0),
+    (700, "ucddcp", 12, 150, 1.0)])
+def test_insert_and_window_moves(lib, move, n, problem, chains, steps, mu, lanes):
+    # insertion (R11b) and contiguous-window (R11c) moves: every chain's trace, best and
+    # final penalty replayed by the oracle; constant temperature keeps many uphill acceptances
+    # (id rotations, best-state copies) in the run
+    if not _lanes_ok(n, lanes):
+        pytest.skip("lanes=4 needs n <= 256")
+    inst = gen.ucddcp_instance(n, 6) if problem == "ucddcp" else gen.cdd_instance(n, 6, 0.4)
+    ins, res, (pen, perm, gid), pr, p, T0 = _run_both(lib, inst, problem, chains, steps, 31 + n,
+                                                     move=move, samples=300, mu=mu, lanes=lanes)
+    tr = res["trace"].cpu().numpy()
+    cb = res["chain_best"].cpu().numpy()
+    cf = res["chain_final"].cpu().numpy()
+    for c in range(chains):
+        ref = oracle.sa_chain(pr, p, T0, c, trace=True)
+        assert np.array_equal(tr[c] >> 1, ref["E_new"]), c
+        assert np.array_equal((tr[c] & 1).astype(bool), ref["accepted"]), c
+        assert cb[c] == ref["E_best"] and cf[c] == ref["E_final"], c
+    full = oracle.sa_run(pr, p, T0)
+    assert (pen, gid) == (full["E_best"], full["g"]) and np.array_equal(perm, full["best"])
+
+
+@pytest.mark.parametrize("move", ["insert", "window"])
+def test_other_moves_no_trace_full_grid(lib, move):
+    # the non-trace kernels (bench configuration) with enough chains for the automatic layout
+    import torch
+
+    inst = gen.cdd_instance(300, 2, 0.6)
+    ins = lib.Instance.from_gen(inst)
+    chains, steps = 4096, 60
+    res = lib.sa_run(ins, chains, steps, move=move, seed=77, T0=500.0, chain_best=True,
+                     chain_final=True)
+    torch.cuda.synchronize()
+    pen, perm, gid = lib.best_get(ins)
+    pr = _prob(inst)
+    p = oracle.sa_params(chains=chains, steps=steps, move=ORACLE_MOVES[move], seed=77)
+    cb = res["chain_best"].cpu().numpy()
+    cf = res["chain_final"].cpu().numpy()
+    for c in list(range(0, chains, 97)) + [chains - 1]:
+        ref = oracle.sa_chain(pr, p, 500.0, c)
+        assert cb[c] == ref["E_best"] and cf[c] == ref["E_final"], c
+    assert oracle.cdd_eval(pr, perm) == pen == cb.min() and gid == int(np.argmin(cb))
 
 
 def test_explicit_T0_and_constant_temperature(lib):

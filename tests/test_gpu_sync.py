@@ -19,19 +19,24 @@ def lib():
     return m
 
 
-def _both(lib, inst, problem, chains, M, levels, seed, lanes=0, T0=0.0, samples=400, mu=0.88):
+MOVES = {"pert_fy": oracle.MOVE_PERT_FY, "insert": oracle.MOVE_INSERT,
+         "window": oracle.MOVE_WINDOW, "swap": oracle.MOVE_SWAP}
+
+
+def _both(lib, inst, problem, chains, M, levels, seed, lanes=0, T0=0.0, samples=400, mu=0.88,
+          move="pert_fy"):
     import torch
 
     ins = lib.Instance.from_gen(inst)
     ss = lib.sa_sync_run(ins, chains, M, levels, problem=problem, seed=seed, lanes=lanes, T0=T0,
-                         t0_samples=samples, mu=mu)
+                         t0_samples=samples, mu=mu, move=move)
     torch.cuda.synchronize()
     pen, perm, gid = lib.best_get(ins)
     pr = oracle.Problem.from_instance(inst)
     P = oracle.CDD if problem == "cdd" else oracle.UCDDCP
     T0_ref = T0 if T0 > 0 else oracle.t0(pr, P, seed, samples)
     assert float(ss.T0.item()) == T0_ref
-    p = oracle.sa_params(problem=P, chains=chains, steps=M, mu=mu, seed=seed)
+    p = oracle.sa_params(problem=P, chains=chains, steps=M, mu=mu, seed=seed, move=MOVES[move])
     ref = oracle.sa_sync(pr, p, T0_ref, levels)
     return ss, (pen, perm, gid), ref
 
@@ -50,6 +55,16 @@ def test_sync_sa_parity(lib, problem, n, chains, M, levels, lanes):
     assert np.array_equal(ss.level_min.cpu().numpy(), ref["level_min_E"])
     assert (pen, gid) == (ref["E_best"], ref["g"])
     assert np.array_equal(perm, ref["best"])
+
+
+@pytest.mark.parametrize("move", ["insert", "window"])
+@pytest.mark.parametrize("problem,n,lanes", [("cdd", 200, 8), ("ucddcp", 90, 4), ("cdd", 1000, 8)])
+def test_sync_sa_other_moves(lib, move, problem, n, lanes):
+    inst = gen.ucddcp_instance(n, 5) if problem == "ucddcp" else gen.cdd_instance(n, 5, 0.4)
+    ss, (pen, perm, gid), ref = _both(lib, inst, problem, 32, 15, 6, seed=3 + n, lanes=lanes,
+                                      move=move)
+    assert np.array_equal(ss.level_min.cpu().numpy(), ref["level_min_E"])
+    assert (pen, gid) == (ref["E_best"], ref["g"]) and np.array_equal(perm, ref["best"])
 
 
 def test_sync_sa_greedy_and_constant_temperature(lib):
