@@ -30,7 +30,7 @@
 extern "C" {
 #endif
 
-#define CDD_ABI_VERSION 4
+#define CDD_ABI_VERSION 5
 
 #if defined(__GNUC__)
 #define CDD_API __attribute__((visibility("default")))
@@ -67,19 +67,30 @@ typedef struct cdd_instance cdd_instance; /* opaque, library-owned, bound to one
 /* Instances (problem data)                                                           */
 /* ------------------------------------------------------------------------------------------ */
 /* Copies the host arrays p, alpha, beta (and m, gamma for UCDDCP; both NULL = CDD only), all
- * indexed by job id, to device `device`.  Checks (CDD_EINVAL): 1 <= n <= 1024, p_i >= 1,
- * alpha_i, beta_i >= 0, 0 <= m_i <= p_i, gamma_i >= 0, d >= 0.  CDD_ERANGE if the data does
- * not fit the packed 32-bit job records of this build (sum alpha, sum beta < 2^16;
- * (sum alpha + sum beta) * sum p < 2^31; field widths for 32 elements per lane <= 32 bits) --
- * always true for the Biskup-Feldmann ranges p<=20, alpha<=10, beta<=15 at n <= 1000.
- * If m/gamma are given but the UCDDCP record (alpha, beta for 32 elements, M, P-M, gamma) does
- * not fit 32 bits, the instance is still created for the CDD and flags bit0 stays clear; the
- * UCDDCP entry points then return CDD_EINVAL.  Synchronous.  *out receives the instance. */
+ * indexed by job id, to device `device`.  The problem data of P:29-49 are general non-negative
+ * integers.  Checks (CDD_EINVAL): 1 <= n <= 32767 (int16 job ids), p_i >= 1, alpha_i, beta_i >= 0,
+ * 0 <= m_i <= p_i, gamma_i >= 0, d >= 0.  CDD_ERANGE only if a penalty could leave the exact
+ * int64 range of the outputs: (sum alpha + sum beta) * sum p + sum gamma * sum (p - m) >= 2^62.
+ *
+ * Fast and generic paths (chosen here, reported by cdd_instance_query flags bit2):
+ *   fast    -- n <= 1024, p <= 255, sum alpha, sum beta < 2^16, (sum alpha + sum beta) * sum p
+ *              < 2^31, 32 * max(alpha, beta) < 2^16 (and for UCDDCP data gamma < 2^16, p - m <=
+ *              255, the packed UCDDCP record fits 32 bits): packed 8/16-bit job records, int32
+ *              arithmetic, the tuned kernels (every Biskup-Feldmann instance, p <= 20, alpha <= 10,
+ *              beta <= 15, at n <= 1000).  The group SA kernels also need alpha, beta <= 255.
+ *   generic -- everything else: int32 fields per job, int64 arithmetic, a warp (n <= 2048) or a
+ *              CTA per sequence.  Serves the batched evaluators, the schedules, asynchronous SA
+ *              (every move) and T0; synchronous SA and DPSO return CDD_EINVAL; the best result is
+ *              read with best_get / best_device_ptrs_wide (best_device_ptrs: CDD_EINVAL).
+ * Both paths compute the same penalties (the closed form of DESIGN.md §4) and draw the same
+ * random numbers, so an instance's results do not depend on the path.  Synchronous.  *out
+ * receives the instance. */
 CDD_API int cdd_instance_create(int32_t n, const int32_t *p, const int32_t *alpha, const int32_t *beta,
                         const int32_t *m, const int32_t *gamma, int64_t d, int device,
                         cdd_instance **out);
 CDD_API int cdd_instance_destroy(cdd_instance *inst);
-/* n, d, sum of p, and flags (bit0: UCDDCP data present, bit1: d >= sum p). Any out may be NULL. */
+/* n, d, sum of p, and flags (bit0: UCDDCP data present, bit1: d >= sum p, bit2: generic path).
+ * Any out may be NULL. */
 CDD_API int cdd_instance_query(const cdd_instance *inst, int32_t *n, int64_t *d, int64_t *sum_p,
                        int32_t *flags);
 
@@ -142,6 +153,7 @@ typedef struct {
     const double *T0_in;   /* optional device double [1]: T0 read on the device (e.g. from sa_t0); */
                            /* overrides T0 / t0_samples when non-NULL                             */
     int32_t lanes;         /* threads per chain: 0 = automatic (by n and chains), 32 = one warp  */
+                           /* per chain (the only layout of the generic path),                   */
                            /* per chain, 4 / 8 / 16 = 8 / 4 / 2 chains per warp (16-bit records: */
                            /* needs alpha, beta <= 255, else CDD_EINVAL); results do not depend  */
                            /* on it (bit-identical), only the speed does                          */
@@ -301,6 +313,11 @@ CDD_API int sa_sync_run_peer(cdd_instance *inst, const sa_sync_params *params, v
  * ties to the lowest id) and int16 [n] sequence.  Valid until the next run or destroy.  The
  * caller may all-reduce the key (MIN) and broadcast the sequence across GPUs in place. */
 CDD_API int best_device_ptrs(cdd_instance *inst, int64_t **packed_dev, int16_t **perm_dev);
+/* Generic-path instances (flags bit2): device int64 [2] = {penalty, global id} and the int16 [n]
+ * sequence (the penalty may exceed the packed key's 32 bits).  Across GPUs: MIN-reduce the
+ * penalty, then the id among the ranks holding that penalty, then broadcast the owner's sequence.
+ * CDD_EINVAL for fast-path instances (use best_device_ptrs).  Added in ABI version 5. */
+CDD_API int best_device_ptrs_wide(cdd_instance *inst, int64_t **pen_id_dev, int16_t **perm_dev);
 /* SYNCHRONOUS: penalty, sequence (host int16 [n], may be NULL) and global chain/particle id. */
 CDD_API int best_get(cdd_instance *inst, int64_t *penalty, int16_t *perm_host, uint64_t *id, void *stream);
 

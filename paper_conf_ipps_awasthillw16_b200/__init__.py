@@ -91,6 +91,7 @@ _SIGS = {
     "dpso_run_peer": (C.c_int, [_vp, C.POINTER(DpsoParams), _vp, _sz, _vp]),
     "sa_sync_run_peer": (C.c_int, [_vp, C.POINTER(SaSyncParams), _vp, _sz, _vp]),
     "best_device_ptrs": (C.c_int, [_vp, _vp, _vp]),
+    "best_device_ptrs_wide": (C.c_int, [_vp, _vp, _vp]),
     "best_get": (C.c_int, [_vp, _vp, _vp, _vp, _vp]),
     "cdd_last_error": (C.c_char_p, []),
     "cdd_abi_version": (C.c_int, []),
@@ -143,6 +144,7 @@ class Instance:
                                         self.d, self.device, C.byref(h)))
         self._h = h
         self.sum_p = int(P.sum())
+        self.wide = self.query()["generic"]
 
     @classmethod
     def from_gen(cls, inst, device=0):
@@ -153,7 +155,7 @@ class Instance:
         n, d, sp, fl = C.c_int32(), C.c_int64(), C.c_int64(), C.c_int32()
         _check(_lib.cdd_instance_query(self.handle, C.byref(n), C.byref(d), C.byref(sp), C.byref(fl)))
         return dict(n=n.value, d=d.value, sum_p=sp.value, has_ucddcp=bool(fl.value & 1),
-                    unrestricted=bool(fl.value & 2))
+                    unrestricted=bool(fl.value & 2), generic=bool(fl.value & 4))
 
     @property
     def handle(self):
@@ -487,6 +489,15 @@ def _device_view(ptr, shape, typestr, device):
     import torch
 
     return torch.as_tensor(_CudaArray(ptr, shape, typestr), device=torch.device("cuda", device))
+
+
+def best_device_tensors_wide(inst: Instance):
+    """Generic-path instances: torch views of the device {penalty, global id} (int64 [2]) and the
+    int16 [n] best sequence."""
+    kp, pp = _vp(), _vp()
+    _check(_lib.best_device_ptrs_wide(inst.handle, C.byref(kp), C.byref(pp)))
+    return (_device_view(kp.value, (2,), "<i8", inst.device),
+            _device_view(pp.value, (inst.n,), "<i2", inst.device))
 
 
 def best_device_tensors(inst: Instance):

@@ -96,6 +96,9 @@ void free_instance(cdd_instance* I) {
     cudaFree(I->tab_m);
     cudaFree(I->tab_x);
     cudaFree(I->tab_g);
+    cudaFree(I->tab_w0);
+    cudaFree(I->tab_w1);
+    cudaFree(I->best_wide);
     cudaFree(I->err);
     cudaFree(I->best_key);
     cudaFree(I->best_perm);
@@ -120,19 +123,37 @@ int cdd_abi_version(void) { return CDD_ABI_VERSION; }
 
 
 
+// The generic path (wide.cu): every array as plain int32 fields by job id, int64 arithmetic.
+static int create_wide(cdd_instance* I, int32_t n, const int32_t* p, const int32_t* alpha,
+                       const int32_t* beta, const int32_t* m, const int32_t* gamma) {
+    std::vector<int4> w0(n);
+    std::vector<int2> w1(m ? n : 0);
+    for (int i = 0; i < n; ++i) {
+        w0[i] = make_int4(p[i], alpha[i], beta[i], gamma ? gamma[i] : 0);
+        if (m) w1[i] = make_int2(m[i], p[i] - m[i]);
+    }
+    cudaError_t e = cudaMalloc(&I->tab_w0, sizeof(int4) * n);
+    if (e == cudaSuccess && m) e = cudaMalloc(&I->tab_w1, sizeof(int2) * n);
+    if (e == cudaSuccess) e = cudaMalloc(&I->best_wide, 2 * sizeof(long long));
+    if (e == cudaSuccess) e = cudaMemcpy(I->tab_w0, w0.data(), sizeof(int4) * n, cudaMemcpyHostToDevice);
+    if (e == cudaSuccess && m) e = cudaMemcpy(I->tab_w1, w1.data(), sizeof(int2) * n, cudaMemcpyHostToDevice);
+    if (e == cudaSuccess) e = cudaMemset(I->best_wide, 0xff, 2 * sizeof(long long));
+    return e == cudaSuccess ? CDD_OK : cuda_fail(e, "cdd_instance_create (generic path)");
+}
+
 int cdd_instance_create(int32_t n, const int32_t* p, const int32_t* alpha, const int32_t* beta,
                         const int32_t* m, const int32_t* gamma, int64_t d, int device,
                         cdd_instance** out) {
     if (!out) return fail(CDD_EINVAL, "out is NULL");
     *out = nullptr;
-    if (n < 1 || n > 1024) return fail(CDD_EINVAL, "n must be in [1, 1024]");
+    if (n < 1 || n > 32767) return fail(CDD_EINVAL, "n must be in [1, 32767] (int16 job ids)");
     if (!p || !alpha || !beta) return fail(CDD_EINVAL, "p, alpha, beta must be non-NULL");
     if ((m == nullptr) != (gamma == nullptr)) return fail(CDD_EINVAL, "m and gamma must both be given or both NULL");
     if (d < 0) return fail(CDD_EINVAL, "d must be >= 0");
     int ndev = 0;
     if (cudaGetDeviceCount(&ndev) != cudaSuccess || device < 0 || device >= ndev)
         return fail(CDD_EINVAL, "invalid CUDA device");
-    int64_t sp = 0, sa = 0, sb = 0;
+    int64_t sp = 0, sa = 0, sb = 0, sg = 0, sx = 0;
     int32_t pmax = 0, amax = 0, bmax = 0, mmax = 0, xmax = 0, gmax = 0;
     for (int i = 0; i < n; ++i) {
         if (p[i] < 1) return fail(CDD_EINVAL, "p_i must be >= 1");
@@ -149,24 +170,66 @@ int cdd_instance_create(int32_t n, const int32_t* p, const int32_t* alpha, const
             mmax = std::max(mmax, m[i]);
             xmax = std::max(xmax, p[i] - m[i]);
             gmax = std::max(gmax, gamma[i]);
+            sg += gamma[i];
+            sx += p[i] - m[i];
         }
     }
-    if (sa >= 65536 || sb >= 65536) return fail(CDD_ERANGE, "sum alpha and sum beta must be < 2^16");
-    if ((sa + sb) * sp >= (int64_t)INT32_MAX) return fail(CDD_ERANGE, "(sum alpha + sum beta) * sum p must be < 2^31");
-    // CDD record: p | a << sa | b << sb, fields wide enough for the sum of 32 records
+    // every penalty of eq. (1) / (2) is at most (sum a + sum b) * sum p (+ sum gamma * sum (p - m));
+    // the outputs are exact int64 below 2^62 (the SA trace packs (E << 1) | accepted)
+    const unsigned __int128 bound = (unsigned __int128)(sa + sb) * (unsigned __int128)sp +
+                                    (unsigned __int128)sg * (unsigned __int128)sx;
+    if (bound >= ((unsigned __int128)1 << 62))
+        return fail(CDD_ERANGE, "penalties could reach 2^62: (sum alpha + sum beta) * sum p + sum gamma * sum (p - m) must be < 2^62");
+    // fast path: packed records (CDD: p | a | b fields wide enough for 32-record lane sums; SA tables:
+    // p, M, P-M bytes, alpha, beta, gamma 16-bit halves) and int32 penalties
     const int wp = bits_for(32ull * (uint64_t)pmax), wa = bits_for(32ull * (uint64_t)amax),
               wb = bits_for(32ull * (uint64_t)bmax);
-    if (wp + wa + wb > 32) return fail(CDD_ERANGE, "p/alpha/beta too large for 32-bit packed records");
-    // warp-per-chain tables: p, M, P-M in bytes; alpha, beta, gamma in 16-bit halves (lane sums of
-    // alpha and beta over 32 positions must stay below 2^16)
-    if (pmax > 255 || 32 * amax >= 65536 || 32 * bmax >= 65536 || gmax >= 65536 || xmax > 255)
-        return fail(CDD_ERANGE, "need p <= 255, alpha, beta < 2048, gamma < 65536 for the SA tables");
+    bool packed = n <= 1024 && sa < 65536 && sb < 65536 && (sa + sb) * sp < (int64_t)INT32_MAX &&
+                  wp + wa + wb <= 32 && pmax <= 255 && 32 * amax < 65536 && 32 * bmax < 65536;
+    int ua = 0, ub = 0, um = 0, ux = 0, ug = 0;
+    if (m) {
+        ua = bits_for(32ull * (uint64_t)amax);
+        ub = bits_for(32ull * (uint64_t)bmax);
+        um = bits_for((uint64_t)mmax);
+        ux = bits_for((uint64_t)xmax);
+        ug = bits_for((uint64_t)gmax);
+        packed = packed && gmax < 65536 && xmax <= 255 && ua + ub + um + ux + ug <= 32;
+    }
     auto* I = new cdd_instance();
     I->device = device;
     I->n = n;
     I->d = d;
     I->sum_p = sp;
     I->d_eff = (int32_t)std::min<int64_t>(d, sp);
+    I->penalty_bound = (int64_t)bound;
+    DeviceGuard g(device);
+    cudaError_t e = cudaSuccess;
+    auto chk = [&](cudaError_t x) {
+        if (e == cudaSuccess) e = x;
+    };
+    chk(cudaMalloc(&I->err, sizeof(int)));
+    chk(cudaMalloc(&I->best_key, sizeof(unsigned long long)));
+    chk(cudaMalloc(&I->best_perm, sizeof(int16_t) * n));
+    if (e == cudaSuccess) {
+        chk(cudaMemset(I->err, 0, sizeof(int)));
+        chk(cudaMemset(I->best_key, 0xff, sizeof(unsigned long long)));
+        chk(cudaMemset(I->best_perm, 0, sizeof(int16_t) * n));
+    }
+    if (e != cudaSuccess) {
+        free_instance(I);
+        return cuda_fail(e, "cdd_instance_create");
+    }
+    if (!packed) {
+        I->wide = true;
+        I->has_ucd = m != nullptr;
+        const int rc = create_wide(I, n, p, alpha, beta, m, gamma);
+        if (rc != CDD_OK) {
+            free_instance(I);
+            return rc;
+        }
+        *out = I;
+        return CDD_OK;
+    }
     I->lay_cdd.sa = wp;
     I->lay_cdd.sb = wp + wa;
     I->lay_cdd.pmask = mask_of(wp);
@@ -176,35 +239,23 @@ int cdd_instance_create(int32_t n, const int32_t* p, const int32_t* alpha, const
     for (int i = 0; i < n; ++i)
         rc[i] = (uint32_t)p[i] | ((uint32_t)alpha[i] << I->lay_cdd.sa) | ((uint32_t)beta[i] << I->lay_cdd.sb);
     if (m) {
-        const int ua = bits_for(32ull * (uint64_t)amax), ub = bits_for(32ull * (uint64_t)bmax);
-        const int um = bits_for((uint64_t)mmax), ux = bits_for((uint64_t)xmax), ug = bits_for((uint64_t)gmax);
-        if (ua + ub + um + ux + ug <= 32) {
-            I->has_ucd = true;
-            auto& L = I->lay_ucd;
-            L.amask = mask_of(ua);
-            L.sb = ua;
-            L.bmask = mask_of(ub);
-            L.sm = ua + ub;
-            L.mmask = mask_of(um);
-            L.sx = L.sm + um;
-            L.xmask = mask_of(ux);
-            L.sg = L.sx + ux;
-            ru.resize(n);
-            for (int i = 0; i < n; ++i)
-                ru[i] = (uint32_t)alpha[i] | ((uint32_t)beta[i] << L.sb) | ((uint32_t)m[i] << L.sm) |
-                        ((uint32_t)(p[i] - m[i]) << L.sx) | ((uint32_t)gamma[i] << L.sg);
-        }  // else: CDD only (flags bit0 clear), the UCDDCP entry points refuse the instance
+        I->has_ucd = true;
+        auto& L = I->lay_ucd;
+        L.amask = mask_of(ua);
+        L.sb = ua;
+        L.bmask = mask_of(ub);
+        L.sm = ua + ub;
+        L.mmask = mask_of(um);
+        L.sx = L.sm + um;
+        L.xmask = mask_of(ux);
+        L.sg = L.sx + ux;
+        ru.resize(n);
+        for (int i = 0; i < n; ++i)
+            ru[i] = (uint32_t)alpha[i] | ((uint32_t)beta[i] << L.sb) | ((uint32_t)m[i] << L.sm) |
+                    ((uint32_t)(p[i] - m[i]) << L.sx) | ((uint32_t)gamma[i] << L.sg);
     }
-    DeviceGuard g(device);
-    cudaError_t e = cudaSuccess;
-    auto chk = [&](cudaError_t x) {
-        if (e == cudaSuccess) e = x;
-    };
     chk(cudaMalloc(&I->rec_cdd, sizeof(uint32_t) * n));
     if (I->has_ucd) chk(cudaMalloc(&I->rec_ucd, sizeof(uint32_t) * n));
-    chk(cudaMalloc(&I->err, sizeof(int)));
-    chk(cudaMalloc(&I->best_key, sizeof(unsigned long long)));
-    chk(cudaMalloc(&I->best_perm, sizeof(int16_t) * n));
     std::vector<uint32_t> tab(n);
     std::vector<uint8_t> tp(n), tm(n), tx(n);
     std::vector<uint16_t> tg(n);
@@ -242,9 +293,6 @@ int cdd_instance_create(int32_t n, const int32_t* p, const int32_t* alpha, const
     if (e == cudaSuccess) {
         chk(cudaMemcpy(I->rec_cdd, rc.data(), sizeof(uint32_t) * n, cudaMemcpyHostToDevice));
         if (I->has_ucd) chk(cudaMemcpy(I->rec_ucd, ru.data(), sizeof(uint32_t) * n, cudaMemcpyHostToDevice));
-        chk(cudaMemset(I->err, 0, sizeof(int)));
-        chk(cudaMemset(I->best_key, 0xff, sizeof(unsigned long long)));
-        chk(cudaMemset(I->best_perm, 0, sizeof(int16_t) * n));
         chk(cdd::probe_smem_base(&I->smem_base));
     }
     if (e != cudaSuccess) {
@@ -266,7 +314,7 @@ int cdd_instance_query(const cdd_instance* I, int32_t* n, int64_t* d, int64_t* s
     if (n) *n = I->n;
     if (d) *d = I->d;
     if (sum_p) *sum_p = I->sum_p;
-    if (flags) *flags = (I->has_ucd ? 1 : 0) | (I->d >= I->sum_p ? 2 : 0);
+    if (flags) *flags = (I->has_ucd ? 1 : 0) | (I->d >= I->sum_p ? 2 : 0) | (I->wide ? 4 : 0);
     return CDD_OK;
 }
 
@@ -279,14 +327,21 @@ static int check_batch_args(const cdd_instance* I, const int16_t* perms, int64_t
     return CDD_OK;
 }
 
+// fast (packed) or generic (wide) evaluator
+static cudaError_t any_eval(const cdd_instance& I, bool ucd, const int16_t* perms, int64_t ld, int64_t batch,
+                            int64_t* out, cudaStream_t s) {
+    return I.wide ? cdd::launch_wide_eval(I, ucd, perms, ld, batch, out, s)
+                  : cdd::launch_eval_batch(I, ucd, perms, ld, batch, out, s);
+}
+
 static int eval_common(cdd_instance* I, bool ucd, const int16_t* perms, int64_t ld, int64_t batch,
                        int64_t* out, void* stream) {
     int rc = check_batch_args(I, perms, ld, batch, out);
     if (rc != CDD_OK) return rc;
-    if (ucd && !I->has_ucd) return fail(CDD_EINVAL, "instance has no UCDDCP data (m/gamma not given or too large for the packed records)");
+    if (ucd && !I->has_ucd) return fail(CDD_EINVAL, "instance has no UCDDCP data (m/gamma not given)");
     if (ucd && I->d < I->sum_p) return fail(CDD_EINVAL, "UCDDCP needs d >= sum p (unrestricted case, P:126)");
     DeviceGuard g(I->device);
-    cudaError_t e = cdd::launch_eval_batch(*I, ucd, perms, ld, batch, out, as_stream(stream));
+    cudaError_t e = any_eval(*I, ucd, perms, ld, batch, out, as_stream(stream));
     return e == cudaSuccess ? CDD_OK : cuda_fail(e, ucd ? "ucddcp_eval_batch" : "cdd_eval_batch");
 }
 
@@ -308,9 +363,10 @@ int cdd_schedule_batch(cdd_instance* I, cdd_problem problem, const int16_t* perm
     if (problem != CDD_PROBLEM_CDD && problem != CDD_PROBLEM_UCDDCP) return fail(CDD_EINVAL, "bad problem");
     const bool ucd = problem == CDD_PROBLEM_UCDDCP;
     if (batch > 0 && (!C || !start || (ucd && !X))) return fail(CDD_EINVAL, "C/start (and X for UCDDCP) must be non-NULL");
-    if (ucd && (!I->has_ucd || I->d < I->sum_p)) return fail(CDD_EINVAL, "instance not usable for UCDDCP (no m/gamma, data too large for the packed records, or d < sum p)");
+    if (ucd && (!I->has_ucd || I->d < I->sum_p)) return fail(CDD_EINVAL, "instance not usable for UCDDCP (no m/gamma, or d < sum p)");
     DeviceGuard g(I->device);
-    cudaError_t e = cdd::launch_schedule(*I, ucd, perms, ld, batch, C, X, start, penalty, as_stream(stream));
+    cudaError_t e = I->wide ? cdd::launch_wide_schedule(*I, ucd, perms, ld, batch, C, X, start, penalty, as_stream(stream))
+                            : cdd::launch_schedule(*I, ucd, perms, ld, batch, C, X, start, penalty, as_stream(stream));
     return e == cudaSuccess ? CDD_OK : cuda_fail(e, "cdd_schedule_batch");
 }
 
@@ -320,7 +376,7 @@ int cdd_eval_batch_host(cdd_instance* I, cdd_problem problem, const int16_t* per
     if (rc != CDD_OK) return rc;
     if (problem != CDD_PROBLEM_CDD && problem != CDD_PROBLEM_UCDDCP) return fail(CDD_EINVAL, "bad problem");
     const bool ucd = problem == CDD_PROBLEM_UCDDCP;
-    if (ucd && (!I->has_ucd || I->d < I->sum_p)) return fail(CDD_EINVAL, "instance not usable for UCDDCP (no m/gamma, data too large for the packed records, or d < sum p)");
+    if (ucd && (!I->has_ucd || I->d < I->sum_p)) return fail(CDD_EINVAL, "instance not usable for UCDDCP (no m/gamma, or d < sum p)");
     DeviceGuard g(I->device);
     cudaStream_t s = as_stream(stream);
     const int64_t chunk = std::max<int64_t>(1, std::min<int64_t>(batch, (int64_t)(256ll << 20) / (ld * 2)));
@@ -339,7 +395,7 @@ int cdd_eval_batch_host(cdd_instance* I, cdd_problem problem, const int16_t* per
         const int64_t rows = std::min(chunk, batch - a);
         cudaError_t e = cudaMemcpyAsync(I->stage_perm, perms_host + a * ld, sizeof(int16_t) * rows * ld,
                                         cudaMemcpyHostToDevice, s);
-        if (e == cudaSuccess) e = cdd::launch_eval_batch(*I, ucd, I->stage_perm, ld, rows, I->stage_out, s);
+        if (e == cudaSuccess) e = any_eval(*I, ucd, I->stage_perm, ld, rows, I->stage_out, s);
         if (e == cudaSuccess)
             e = cudaMemcpyAsync(out_host + a, I->stage_out, sizeof(int64_t) * rows, cudaMemcpyDeviceToHost, s);
         if (e != cudaSuccess) return cuda_fail(e, "cdd_eval_batch_host");
@@ -369,7 +425,7 @@ static int sa_validate(const cdd_instance* I, const sa_params* p, cdd::SaLaunch*
     if (!I || !p) return fail(CDD_EINVAL, "instance/params is NULL");
     if (p->problem != CDD_PROBLEM_CDD && p->problem != CDD_PROBLEM_UCDDCP) return fail(CDD_EINVAL, "bad problem");
     const bool ucd = p->problem == CDD_PROBLEM_UCDDCP;
-    if (ucd && (!I->has_ucd || I->d < I->sum_p)) return fail(CDD_EINVAL, "instance not usable for UCDDCP (no m/gamma, data too large for the packed records, or d < sum p)");
+    if (ucd && (!I->has_ucd || I->d < I->sum_p)) return fail(CDD_EINVAL, "instance not usable for UCDDCP (no m/gamma, or d < sum p)");
     if (p->chains < 1) return fail(CDD_EINVAL, "chains must be >= 1");
     if (p->steps < 0 || p->steps >= (int64_t)UINT32_MAX) return fail(CDD_EINVAL, "steps must be in [0, 2^32)");
     if (p->chain_offset + (uint64_t)p->chains > (1ull << 32)) return fail(CDD_EINVAL, "chain ids must fit 32 bits");
@@ -383,7 +439,10 @@ static int sa_validate(const cdd_instance* I, const sa_params* p, cdd::SaLaunch*
     if (p->lanes != 0 && p->lanes != 4 && p->lanes != 8 && p->lanes != 16 && p->lanes != 32)
         return fail(CDD_EINVAL, "lanes must be 0, 4, 8, 16 or 32");
     if (p->lanes >= 4 && p->lanes <= 16 && !I->ab16_ok)
-        return fail(CDD_EINVAL, "lanes 4/8/16 need alpha, beta <= 255 (16-bit records)");
+        return fail(CDD_EINVAL, "lanes 4/8/16 need alpha, beta <= 255 (16-bit records, fast path)");
+    if (I->wide && !(p->T0 > 0) && !p->T0_in &&
+        (unsigned __int128)p->t0_samples * (unsigned __int128)(uint64_t)I->penalty_bound >= ((unsigned __int128)1 << 65))
+        return fail(CDD_EINVAL, "T0 from samples: t0_samples * penalty bound must be < 2^65 (exact 128-bit moments); give T0");
     if (p->lanes == 4 && I->n > 256) return fail(CDD_EINVAL, "lanes = 4 supports n <= 256");
     if (p->init && p->init_ld != 0 && p->init_ld < I->n) return fail(CDD_EINVAL, "init_ld must be 0 or >= n");
     L->ucd = ucd;
@@ -411,7 +470,7 @@ size_t sa_workspace_size(const cdd_instance* I, const sa_params* p) {
     cdd::SaLaunch L{};
     if (sa_validate(I, p, &L) != CDD_OK) return 0;
     DeviceGuard g(I->device);
-    return cdd::sa_workspace_bytes(*I, L);
+    return I->wide ? cdd::wide_sa_workspace_bytes(*I, L) : cdd::sa_workspace_bytes(*I, L);
 }
 
 static int sync_validate(const cdd_instance* I, const sa_sync_params* q, cdd::SaLaunch* L) {
@@ -421,7 +480,7 @@ static int sync_validate(const cdd_instance* I, const sa_sync_params* q, cdd::Sa
         return fail(CDD_EINVAL, "levels * markov_len must be < 2^32");
     if (q->lanes != 0 && q->lanes != 4 && q->lanes != 8 && q->lanes != 16)
         return fail(CDD_EINVAL, "synchronous SA runs on lanes 0, 4, 8 or 16");
-    if (!I->ab16_ok) return fail(CDD_EINVAL, "synchronous SA needs alpha, beta <= 255 (16-bit records)");
+    if (!I->ab16_ok) return fail(CDD_EINVAL, "synchronous SA needs the fast path (packed records, alpha, beta <= 255)");
     sa_params p{};
     p.problem = q->problem;
     p.chains = q->chains;
@@ -468,9 +527,9 @@ int sa_sync_run_peer(cdd_instance* I, const sa_sync_params* q, void* ws, size_t 
     if (rc != CDD_OK) return rc;
     cdd::DpsoPeer* P = I->peer;
     if (!P || !P->open) return fail(CDD_ESTATE, "peer exchange not open (dpso_peer_create / dpso_peer_open)");
-    if (!P->armed) return fail(CDD_ESTATE, "peer exchange not re-armed: dpso_peer_reset (+ a barrier) before every fused run");
     if (q->chain_offset != (uint64_t)P->rank * (uint64_t)q->chains)
         return fail(CDD_EINVAL, "chain_offset must be rank * chains (equal shares)");
+    if (!P->armed) return fail(CDD_ESTATE, "peer exchange not re-armed: dpso_peer_reset (+ a barrier) before every fused run");
     DeviceGuard g(I->device);
     const size_t need = cdd::sa_sync_workspace_bytes(*I, L);
     if (!ws || ws_bytes < need)
@@ -523,10 +582,10 @@ int sa_run(cdd_instance* I, const sa_params* p, void* ws, size_t ws_bytes, void*
     int rc = sa_validate(I, p, &L);
     if (rc != CDD_OK) return rc;
     DeviceGuard g(I->device);
-    const size_t need = cdd::sa_workspace_bytes(*I, L);
+    const size_t need = I->wide ? cdd::wide_sa_workspace_bytes(*I, L) : cdd::sa_workspace_bytes(*I, L);
     if (!ws || ws_bytes < need)
         return fail(CDD_ENOMEM, "workspace too small: need " + std::to_string(need) + " bytes");
-    cudaError_t e = cdd::launch_sa(*I, L, ws, as_stream(stream));
+    cudaError_t e = I->wide ? cdd::launch_wide_sa(*I, L, ws, as_stream(stream)) : cdd::launch_sa(*I, L, ws, as_stream(stream));
     if (e != cudaSuccess) return cuda_fail(e, "sa_run");
     I->has_best = true;
     return CDD_OK;
@@ -548,10 +607,11 @@ int sa_t0(cdd_instance* I, cdd_problem problem, uint64_t seed, int64_t samples, 
     int rc = sa_validate(I, &p, &L);
     if (rc != CDD_OK) return rc;
     DeviceGuard g(I->device);
-    const size_t need = cdd::sa_workspace_bytes(*I, L);
+    const size_t need = I->wide ? cdd::wide_sa_workspace_bytes(*I, L) : cdd::sa_workspace_bytes(*I, L);
     if (!ws || ws_bytes < need)
         return fail(CDD_ENOMEM, "workspace too small: need " + std::to_string(need) + " bytes");
-    cudaError_t e = cdd::launch_t0(*I, L.ucd, seed, samples, T0_dev, ws, as_stream(stream));
+    cudaError_t e = I->wide ? cdd::launch_wide_t0(*I, L.ucd, seed, samples, T0_dev, ws, as_stream(stream))
+                            : cdd::launch_t0(*I, L.ucd, seed, samples, T0_dev, ws, as_stream(stream));
     return e == cudaSuccess ? CDD_OK : cuda_fail(e, "sa_t0");
 }
 
@@ -559,8 +619,9 @@ static int dpso_validate(const cdd_instance* I, const dpso_params* p, cdd::DpsoL
     if (!I || !p) return fail(CDD_EINVAL, "instance/params is NULL");
     if (p->problem != CDD_PROBLEM_CDD && p->problem != CDD_PROBLEM_UCDDCP) return fail(CDD_EINVAL, "bad problem");
     const bool ucd = p->problem == CDD_PROBLEM_UCDDCP;
-    if (ucd && (!I->has_ucd || I->d < I->sum_p)) return fail(CDD_EINVAL, "instance not usable for UCDDCP (no m/gamma, data too large for the packed records, or d < sum p)");
+    if (ucd && (!I->has_ucd || I->d < I->sum_p)) return fail(CDD_EINVAL, "instance not usable for UCDDCP (no m/gamma, or d < sum p)");
     if (I->n < 2) return fail(CDD_EINVAL, "DPSO needs n >= 2");
+    if (I->wide) return fail(CDD_EINVAL, "DPSO runs on the fast path only (packed records: n <= 1024, p <= 255, ...)");
     if (p->particles < 1 || p->particles >= (1ll << 31)) return fail(CDD_EINVAL, "particles must be in [1, 2^31)");
     if (p->iters < 0 || p->iters >= (int64_t)UINT32_MAX) return fail(CDD_EINVAL, "iters must be in [0, 2^32)");
     if (p->particle_offset + (uint64_t)p->particles > (1ull << 32)) return fail(CDD_EINVAL, "particle ids must fit 32 bits");
@@ -748,11 +809,11 @@ int dpso_run_peer(cdd_instance* I, const dpso_params* p, void* ws, size_t ws_byt
     if (rc != CDD_OK) return rc;
     cdd::DpsoPeer* P = I->peer;
     if (!P || !P->open) return fail(CDD_ESTATE, "peer exchange not open (dpso_peer_create / dpso_peer_open)");
-    if (!P->armed) return fail(CDD_ESTATE, "peer exchange not re-armed: dpso_peer_reset (+ a barrier) before every fused run");
     if (p->particle_offset != (uint64_t)P->rank * (uint64_t)p->particles)
         return fail(CDD_EINVAL, "particle_offset must be rank * particles (equal shares)");
     if ((uint64_t)p->particles * (uint64_t)P->world > (1ull << 32))
         return fail(CDD_EINVAL, "global particle ids must fit 32 bits");
+    if (!P->armed) return fail(CDD_ESTATE, "peer exchange not re-armed: dpso_peer_reset (+ a barrier) before every fused run");
     L.peer = true;
     P->armed = false;
     DeviceGuard g(I->device);
@@ -767,7 +828,16 @@ int dpso_run_peer(cdd_instance* I, const dpso_params* p, void* ws, size_t ws_byt
 
 int best_device_ptrs(cdd_instance* I, int64_t** packed_dev, int16_t** perm_dev) {
     if (!I) return fail(CDD_EINVAL, "instance is NULL");
+    if (I->wide) return fail(CDD_EINVAL, "generic-path instance: penalties may exceed the packed key, use best_device_ptrs_wide");
     if (packed_dev) *packed_dev = reinterpret_cast<int64_t*>(I->best_key);
+    if (perm_dev) *perm_dev = I->best_perm;
+    return CDD_OK;
+}
+
+int best_device_ptrs_wide(cdd_instance* I, int64_t** pen_id_dev, int16_t** perm_dev) {
+    if (!I) return fail(CDD_EINVAL, "instance is NULL");
+    if (!I->wide) return fail(CDD_EINVAL, "fast-path instance: use best_device_ptrs (packed key)");
+    if (pen_id_dev) *pen_id_dev = reinterpret_cast<int64_t*>(I->best_wide);
     if (perm_dev) *perm_dev = I->best_perm;
     return CDD_OK;
 }
@@ -778,11 +848,19 @@ int best_get(cdd_instance* I, int64_t* penalty, int16_t* perm_host, uint64_t* id
     DeviceGuard g(I->device);
     cudaStream_t s = as_stream(stream);
     unsigned long long key = 0;
-    cudaError_t e = cudaMemcpyAsync(&key, I->best_key, sizeof key, cudaMemcpyDeviceToHost, s);
+    long long pw[2] = {-1, -1};
+    cudaError_t e = I->wide ? cudaMemcpyAsync(pw, I->best_wide, sizeof pw, cudaMemcpyDeviceToHost, s)
+                            : cudaMemcpyAsync(&key, I->best_key, sizeof key, cudaMemcpyDeviceToHost, s);
     if (e == cudaSuccess && perm_host)
         e = cudaMemcpyAsync(perm_host, I->best_perm, sizeof(int16_t) * I->n, cudaMemcpyDeviceToHost, s);
     if (e == cudaSuccess) e = cudaStreamSynchronize(s);
     if (e != cudaSuccess) return cuda_fail(e, "best_get");
+    if (I->wide) {
+        if (pw[0] < 0 || pw[0] == LLONG_MAX) return fail(CDD_ESTATE, "no result");
+        if (penalty) *penalty = pw[0];
+        if (id) *id = (uint64_t)pw[1];
+        return CDD_OK;
+    }
     if (key == ULLONG_MAX) return fail(CDD_ESTATE, "no result");
     if (penalty) *penalty = (int64_t)(key >> 32);
     if (id) *id = key & 0xffffffffull;

@@ -55,6 +55,12 @@ struct Instance {
     uint8_t* tab_m = nullptr;
     uint8_t* tab_x = nullptr;
     uint16_t* tab_g = nullptr;
+    // generic ("wide") path (wide.cu): instances outside the packed record ranges
+    bool wide = false;
+    int64_t penalty_bound = 0;  // (sum a + sum b) * sum p + sum gamma * sum (P - M) (< 2^62)
+    int4* tab_w0 = nullptr;  // {P, alpha, beta, gamma} by job id
+    int2* tab_w1 = nullptr;  // {M, P - M} by job id (UCDDCP)
+    long long* best_wide = nullptr;  // device {penalty, global id} of the last run (wide instances)
     int* err = nullptr;                    // device data-error flag
     unsigned long long* best_key = nullptr;  // device packed (penalty << 32 | id)
     int16_t* best_perm = nullptr;          // device [n]
@@ -135,6 +141,16 @@ cudaError_t dpso_iterate(Instance& I, const DpsoLaunch& p, void* ws, int64_t t0,
 void dpso_gbest(const Instance& I, const DpsoLaunch& p, void* ws, int64_t t, int64_t** key,
                 int16_t** perm);
 cudaError_t dpso_end(Instance& I, const DpsoLaunch& p, void* ws, cudaStream_t s);
+
+// ---- launchers (wide.cu): the generic path (int64, n <= 32767, no packing)
+cudaError_t launch_wide_eval(const Instance& I, bool ucd, const int16_t* perms, int64_t ld, int64_t batch,
+                             int64_t* out, cudaStream_t s);
+cudaError_t launch_wide_schedule(const Instance& I, bool ucd, const int16_t* perms, int64_t ld, int64_t batch,
+                                 int64_t* C, int32_t* X, int64_t* start, int64_t* pen, cudaStream_t s);
+size_t wide_sa_workspace_bytes(const Instance& I, const SaLaunch& p);
+cudaError_t launch_wide_t0(const Instance& I, bool ucd, uint64_t seed, int64_t samples, double* T0_dev, void* ws,
+                           cudaStream_t s);
+cudaError_t launch_wide_sa(Instance& I, const SaLaunch& p, void* ws, cudaStream_t s);
 
 int sa_e_for_n(int n);  // elements per lane of the warp-per-chain kernels
 

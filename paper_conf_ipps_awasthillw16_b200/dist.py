@@ -77,8 +77,35 @@ def reduce_best_async(key: torch.Tensor, perm: torch.Tensor, group=None) -> None
     dist.all_reduce(perm.view(torch.uint8), op=dist.ReduceOp.SUM, group=group)
 
 
+def reduce_best_wide(pen_id: torch.Tensor, perm: torch.Tensor, group=None) -> None:
+    """Generic-path instances (penalties beyond the packed key): pen_id = int64 [2] {penalty, global
+    id}, empty = {-1, -1}.  In place: the lexicographic minimum over ranks and the owner's sequence
+    -- MIN of the penalty, MIN of the id among the ranks holding it, then a SUM of the sequences
+    with every non-owner's zeroed (no host round trip)."""
+    pen, gid = pen_id[0:1].clone(), pen_id[1:2].clone()
+    empty = pen < 0
+    pen.masked_fill_(empty, _INT64_MAX)
+    p = pen.clone()
+    dist.all_reduce(p, op=dist.ReduceOp.MIN, group=group)
+    g = torch.where((pen == p) & ~empty, gid, torch.full_like(gid, _INT64_MAX))
+    dist.all_reduce(g, op=dist.ReduceOp.MIN, group=group)
+    mine = (pen == p) & (gid == g) & ~empty
+    perm.mul_(mine.to(perm.dtype))
+    dist.all_reduce(perm.view(torch.uint8), op=dist.ReduceOp.SUM, group=group)
+    none = p == _INT64_MAX
+    pen_id[0:1].copy_(torch.where(none, torch.full_like(p, -1), p))
+    pen_id[1:2].copy_(torch.where(none, torch.full_like(g, -1), g))
+
+
 def global_best(inst, ids_per_rank: int, group=None) -> int:
-    """Reduce the instance's device-resident best (after sa_run / dpso_run) across all ranks."""
+    """Reduce the instance's device-resident best (after sa_run / dpso_run) across all ranks.
+    Returns the owner's rank (fast path; -1 without a result; generic path: -2, not computed)."""
+    if getattr(inst, "wide", False):
+        from . import best_device_tensors_wide
+
+        pen_id, perm = best_device_tensors_wide(inst)
+        reduce_best_wide(pen_id, perm, group)
+        return -2
     key, perm = best_device_tensors(inst)
     return reduce_best(key, perm, ids_per_rank, group)
 
@@ -86,6 +113,12 @@ def global_best(inst, ids_per_rank: int, group=None) -> int:
 def global_best_async(inst, group=None) -> None:
     """global_best without the host round trip (reduce_best_async on the best buffers): the next
     run's launches queue behind the collectives instead of waiting for them."""
+    if getattr(inst, "wide", False):
+        from . import best_device_tensors_wide
+
+        pen_id, perm = best_device_tensors_wide(inst)
+        reduce_best_wide(pen_id, perm, group)
+        return
     key, perm = best_device_tensors(inst)
     reduce_best_async(key, perm, group)
 

@@ -136,6 +136,9 @@ def test_peer_exchange_api_single_rank(lib):
     with pytest.raises(lib.CddError) as e:
         bad.run_peer()  # particle_offset must be rank * particles
     assert e.value.code == lib.CDD_EINVAL
+    with pytest.raises(lib.CddError) as e:
+        sw.run_peer()  # a second fused run without dpso_peer_reset
+    assert e.value.code == lib.CDD_ESTATE
     # synchronous SA through the same exchange
     lib.dpso_peer_reset(ins)
     ss = lib.SaSync(ins, 2048, 6, 4, seed=9, t0_samples=300).run_peer()
