@@ -43,6 +43,18 @@ def _peaks():
         return {}
 
 
+def _int_peak():
+    """Best measured integer rate of this GPU model (scripts/int_peak.cu, committed measurements)."""
+    best = {"op": "nominal 4 SMSP x 32 lanes", "lane_ops_per_clk_per_sm": 128.0,
+            "warp_instr_per_clk_per_sm": 4.0}
+    path = os.path.join(ROOT, "profiles", "r2_int_peak.jsonl")
+    if os.path.exists(path):
+        rows = [json.loads(x) for x in open(path) if x.strip().startswith("{")]
+        if rows:
+            best = max(rows, key=lambda r: r["lane_ops_per_clk_per_sm"])
+    return best
+
+
 def _evals_per_step(chains, steps, samples, instances):
     return instances * (samples + chains * (steps + 1))
 
@@ -146,18 +158,35 @@ def run_reference(args):
     print(json.dumps(line), flush=True)
 
 
+def _cpu_model():
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return None
+
+
 def cpu_baseline_sample(seconds=12.0):
-    """Oracle SA timed on the host cores (bounded sample of the same workload)."""
+    """Oracle SA timed on the host cores (bounded sample of the same workload), plus the oracle's
+    single-thread rate and its batched-evaluation rate (BASELINE.md's CPU-baseline plan)."""
     import gen
+    import numpy as np
     import oracle
 
     threads = os.cpu_count() or 1
-    pr = oracle.Problem.from_instance(gen.cdd_instance(N_JOBS, INSTANCE_SEED, 0.4))
+    inst = gen.cdd_instance(N_JOBS, INSTANCE_SEED, 0.4)
+    pr = oracle.Problem.from_instance(inst)
     T0 = oracle.t0(pr, oracle.CDD, RUN_SEED, 200)
-    # size the per-thread chain so the sample takes about `seconds`
+    # single thread: one chain for ~2 s; sizes the per-thread chain of the all-core sample
     t = time.perf_counter()
     oracle.sa_chain(pr, oracle.sa_params(steps=200, seed=RUN_SEED), T0, 0)
     per_eval = (time.perf_counter() - t) / 201
+    st_steps = max(50, int(2.0 / per_eval))
+    t = time.perf_counter()
+    oracle.sa_chain(pr, oracle.sa_params(steps=st_steps, seed=RUN_SEED), T0, 1)
+    single = (st_steps + 1) / (time.perf_counter() - t)
     steps = max(50, int(seconds / per_eval))
     done = [0]
 
@@ -170,9 +199,18 @@ def cpu_baseline_sample(seconds=12.0):
     [x.start() for x in ts]
     [x.join() for x in ts]
     dt = time.perf_counter() - t
+    # batched evaluation (the cdd_eval_batch leg's workload: random sequences at n=1000), ~3 s
+    rows = max(threads, int(3.0 / per_eval) * threads)
+    perms = gen.random_perms(rows, N_JOBS, 7, ld=N_JOBS)
+    t = time.perf_counter()
+    oracle.eval_batch_threaded(pr, perms, threads=threads)
+    ev_rate = rows / (time.perf_counter() - t)
     return {"value": done[0] / dt, "unit": "evals/s", "cores": threads, "kind": "oracle",
+            "cpu_model": _cpu_model(), "single_thread_evals_per_s": single,
+            "eval_batch_evals_per_s": ev_rate,
             "sample": f"{threads} host threads x 1 SA chain x {steps} steps, CDD n=1000 h=0.4 "
-                      f"(T0 from 200 samples, excluded); {dt:.1f} s"}
+                      f"(T0 from 200 samples, excluded); {dt:.1f} s; single thread {st_steps} steps; "
+                      f"batched evaluation of {rows} random sequences on {threads} threads"}
 
 
 # ------------------------------------------------------------------------------ GPU arm
@@ -283,15 +321,20 @@ def main():
             entry["gap_pct"] = 100.0 * (pen - ref) / ref
         gaps[key] = entry
 
-    # roofline of the dominant kernel (sa_kernel): algorithmic int ops / its event duration
+    # roofline of the dominant kernel (sa_group_kernel): algorithmic int ops / its event duration,
+    # against the MEASURED integer peak of this B200 (scripts/int_peak.cu -> profiles/r2_int_peak.jsonl:
+    # the best lane-op rate of the measured opcode mixes), plus the issue view (ncu-counted warp
+    # instructions per evaluation / measured best warp-instruction rate)
     peaks = _peaks()
     sm_max = float(peaks.get("sm_max_mhz", 1965.0))
     kms = [a.elapsed_time(b) for a, b in kernel_ev]
     k_avg_ms = sum(kms) / len(kms)
-    ops = INT_OPS_PER_ELEM * N_JOBS * chains * (steps + 1)
+    evals_launch = chains * (steps + 1)
+    ops = INT_OPS_PER_ELEM * N_JOBS * evals_launch
     achieved = ops / (k_avg_ms / 1000.0) / 1e12
     nsm = torch.cuda.get_device_properties(dev).multi_processor_count
-    peak = 128 * nsm * sm_max * 1e6 / 1e12
+    ip = _int_peak()
+    peak = ip["lane_ops_per_clk_per_sm"] * nsm * sm_max * 1e6 / 1e12
     traffic = None
     tp = os.path.join(ROOT, "profiles", "sa_kernel_dram_bytes.json")
     if os.path.exists(tp):
@@ -300,11 +343,24 @@ def main():
     G, E = lib.sa_layout(insts[0], chains)
     kname = (f"sa_group_kernel<{G},{E}> (CDD, {32 // G} chains per warp)" if G < 32
              else f"sa_kernel<{E}> (CDD, one warp per chain)")
+    issue = None
+    ipath = os.path.join(ROOT, "profiles", "sa_kernel_issue.json")
+    if os.path.exists(ipath):
+        ipe = json.load(open(ipath))["warp_instr_per_eval"]
+        rate = ipe * evals_launch / (k_avg_ms / 1000.0) / (nsm * sm_max * 1e6)
+        issue = {"warp_instr_per_eval": ipe, "achieved_warp_instr_per_clk_per_sm": rate,
+                 "peak_warp_instr_per_clk_per_sm": ip["warp_instr_per_clk_per_sm"],
+                 "frac": rate / ip["warp_instr_per_clk_per_sm"],
+                 "note": "instructions per evaluation from ncu (profiles/sa_kernel_issue.json); peak = best "
+                         "measured issue rate (profiles/r2_int_peak.jsonl); at max SM clock"}
     roofline = {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "Tint-op/s",
                 "frac": achieved / peak, "traffic": traffic, "kernel": kname,
                 "kernel_ms_avg": k_avg_ms, "kernel_share_of_step": k_avg_ms * len(insts) / step_ms,
-                "ops_per_launch": ops,
-                "peak_note": f"128 int32 lane-ops/clk/SM (4 SMSP x 32 lanes issue, alu+fma pipes) x {nsm} SMs x {sm_max:.0f} MHz max clock"}
+                "ops_per_launch": ops, "issue": issue,
+                "peak_note": (f"measured: {ip['lane_ops_per_clk_per_sm']:.1f} int32 lane-ops/clk/SM "
+                              f"({ip['op']}, scripts/int_peak.cu, profiles/r2_int_peak.jsonl) x {nsm} SMs x "
+                              f"{sm_max:.0f} MHz max clock; algorithmic ops = {INT_OPS_PER_ELEM}n per evaluation "
+                              f"(SURVEY 8(d))")}
 
     extra = {}
     if rank == 0 and not args.no_eval:
@@ -319,7 +375,7 @@ def main():
     if not args.no_e2e:
         e2e = bench_e2e(lib, gens, chains, steps, rank, world, dev, stream, max(1, args.steps // 2))
     cpu = None
-    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+    if rank == 0 and not args.no_cpu_baseline:  # after the timed region (also at N > 1)
         cpu = cpu_baseline_sample()
 
     if rank == 0:

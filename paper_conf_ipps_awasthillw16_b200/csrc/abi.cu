@@ -35,7 +35,16 @@ void resident_ctas(const void* kern, int device, int threads, size_t smem, int* 
     }
     int s = 148, o = 1;
     cudaDeviceGetAttribute(&s, cudaDevAttrMultiProcessorCount, device);
-    cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    {
+        // the dynamic-smem attribute only ever grows: a launch shape memoised earlier must stay valid
+        static std::map<std::pair<const void*, int>, size_t> attr;
+        std::lock_guard<std::mutex> lk(mu);
+        size_t& cur = attr[std::make_pair(kern, device)];
+        if (smem > cur) {
+            cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+            cur = smem;
+        }
+    }
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, kern, threads, smem);
     if (o < 1) o = 1;
     *sms = s;
@@ -720,7 +729,7 @@ int dpso_peer_create(cdd_instance* I, int world, int rank, uint8_t* ipc_handle) 
     auto* P = new cdd::DpsoPeer();
     P->world = world;
     P->rank = rank;
-    P->np = 32 * cdd::sa_e_for_n(I->n);
+    P->np = cdd::dpso_np(I->n);
     const size_t bytes = cdd::dpso_peer_region_bytes(I->n);
     cudaError_t e = cudaMalloc(&P->region, bytes);
     if (e == cudaSuccess) e = cudaMemset(P->region, 0, bytes);

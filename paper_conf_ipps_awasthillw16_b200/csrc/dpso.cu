@@ -15,6 +15,7 @@
 #include <cuda_runtime.h>
 
 #include <climits>
+#include <cstdlib>
 
 #include "chain.cuh"
 #include "device_common.cuh"
@@ -446,18 +447,20 @@ constexpr size_t kAlign = 256;
 inline size_t align_up(size_t x) { return (x + kAlign - 1) / kAlign * kAlign; }
 
 struct DpWs {
-    size_t pos, pb, zb, gkey, gperm, counter, total;
+    size_t pos, inv, pb, zb, gkey, gperm, counter, ctakeys, total;
 };
 
 DpWs dp_layout(int np, int64_t N) {
     DpWs w{};
     w.pos = 0;
-    w.pb = align_up(w.pos + (size_t)N * np * 2);
+    w.inv = align_up(w.pos + (size_t)N * np * 2);
+    w.pb = align_up(w.inv + (size_t)N * np * 2);
     w.zb = align_up(w.pb + (size_t)N * np * 2);
     w.gkey = align_up(w.zb + (size_t)N * 4);
     w.gperm = align_up(w.gkey + 16);
     w.counter = align_up(w.gperm + (size_t)2 * np * 2);
-    w.total = align_up(w.counter + 16);
+    w.ctakeys = align_up(w.counter + 16);
+    w.total = align_up(w.ctakeys + sizeof(unsigned long long) * kDpsoMaxCtas);
     return w;
 }
 
@@ -466,10 +469,28 @@ ChainTables dp_tables(const Instance& I, bool ucd) {
                : ChainTables{I.tab_ab, I.tab_p, nullptr, nullptr, I.ab16_ok ? I.tab_ab16 : nullptr};
 }
 
+DpsoWsPtrs ws_ptrs(const Instance& I, const DpsoLaunch& p, void* ws) {
+    const int np = dpso_np(I.n);
+    const DpWs w = dp_layout(np, p.particles);
+    uint8_t* b = static_cast<uint8_t*>(ws);
+    DpsoWsPtrs r{};
+    r.pos = reinterpret_cast<int16_t*>(b + w.pos);
+    r.inv = reinterpret_cast<int16_t*>(b + w.inv);
+    r.pb = reinterpret_cast<int16_t*>(b + w.pb);
+    r.zb = reinterpret_cast<int32_t*>(b + w.zb);
+    r.gkey = reinterpret_cast<unsigned long long*>(b + w.gkey);
+    r.gperm = reinterpret_cast<int16_t*>(b + w.gperm);
+    r.counter = reinterpret_cast<unsigned int*>(b + w.counter);
+    r.ctakeys = reinterpret_cast<unsigned long long*>(b + w.ctakeys);
+    r.np = np;
+    return r;
+}
+
+bool use_group(const Instance& I) { return dpsog_usable(I); }
+
 template <int E>
 DpArgs make_args(const Instance& I, const DpsoLaunch& p, void* ws) {
-    constexpr int NP = 32 * E;
-    const DpWs w = dp_layout(NP, p.particles);
+    const DpWs w = dp_layout(dpso_np(I.n), p.particles);
     uint8_t* b = static_cast<uint8_t*>(ws);
     DpArgs a{};
     a.T = dp_tables(I, p.ucd);
@@ -495,7 +516,7 @@ DpArgs make_args(const Instance& I, const DpsoLaunch& p, void* ws) {
         a.pregions = I.peer->d_regions;
     }
     a.trace = p.gbest_trace;
-    a.np = NP;
+    a.np = dpso_np(I.n);
     return a;
 }
 
@@ -562,13 +583,14 @@ cudaError_t iter_d(Instance& I, const DpsoLaunch& p, void* ws, int64_t t0, int64
 
 }  // namespace
 
-size_t dpso_peer_region_bytes(int n) { return kPeerPermOff + (size_t)2 * 32 * sa_e_for_n(n) * sizeof(int16_t); }
+size_t dpso_peer_region_bytes(int n) { return kPeerPermOff + (size_t)2 * dpso_np(n) * sizeof(int16_t); }
 
 size_t dpso_workspace_bytes(const Instance& I, const DpsoLaunch& p) {
-    return dp_layout(32 * sa_e_for_n(I.n), p.particles).total;
+    return dp_layout(dpso_np(I.n), p.particles).total;
 }
 
 cudaError_t dpso_begin(Instance& I, const DpsoLaunch& p, void* ws, cudaStream_t s) {
+    if (use_group(I)) return dpsog_begin(I, p, ws_ptrs(I, p, ws), s);
     switch (sa_e_for_n(I.n)) {
         case 1: return begin_d<1>(I, p, ws, s);
         case 2: return begin_d<2>(I, p, ws, s);
@@ -581,6 +603,7 @@ cudaError_t dpso_begin(Instance& I, const DpsoLaunch& p, void* ws, cudaStream_t 
 
 cudaError_t dpso_iterate(Instance& I, const DpsoLaunch& p, void* ws, int64_t t0, int64_t t1,
                          cudaStream_t s) {
+    if (use_group(I)) return dpsog_iterate(I, p, ws_ptrs(I, p, ws), t0, t1, s);
     switch (sa_e_for_n(I.n)) {
         case 1: return iter_d<1>(I, p, ws, t0, t1, s);
         case 2: return iter_d<2>(I, p, ws, t0, t1, s);
@@ -593,7 +616,7 @@ cudaError_t dpso_iterate(Instance& I, const DpsoLaunch& p, void* ws, int64_t t0,
 
 void dpso_gbest(const Instance& I, const DpsoLaunch& p, void* ws, int64_t t, int64_t** key,
                 int16_t** perm) {
-    const int np = 32 * sa_e_for_n(I.n);
+    const int np = dpso_np(I.n);
     const DpWs w = dp_layout(np, p.particles);
     uint8_t* b = static_cast<uint8_t*>(ws);
     const int par = (int)(t & 1);

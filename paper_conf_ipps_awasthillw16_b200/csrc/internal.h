@@ -133,6 +133,23 @@ struct DpsoLaunch {
     bool peer = false;  // exchange the swarm best through Instance::peer inside the kernels
 };
 size_t dpso_peer_region_bytes(int n);
+int dpso_np(int n);  // row stride of the DPSO workspace and of the peer regions
+// workspace of a DPSO run (dpso.cu dp_layout), shared by both kernel layouts
+struct DpsoWsPtrs {
+    int16_t *pos, *inv, *pb;
+    int32_t* zb;
+    unsigned long long* gkey;
+    int16_t* gperm;
+    unsigned int* counter;
+    unsigned long long* ctakeys;  // per-CTA minimum keys (group layout's publish), kDpsoMaxCtas
+    int np;
+};
+constexpr int kDpsoMaxCtas = 8192;
+// group-layout DPSO (dpso_group.cu): 8 lanes per particle; needs the 16-bit records (ab16_ok)
+bool dpsog_usable(const Instance& I);
+cudaError_t dpsog_begin(Instance& I, const DpsoLaunch& p, const DpsoWsPtrs& w, cudaStream_t s);
+cudaError_t dpsog_iterate(Instance& I, const DpsoLaunch& p, const DpsoWsPtrs& w, int64_t t0, int64_t t1,
+                          cudaStream_t s);
 size_t dpso_workspace_bytes(const Instance& I, const DpsoLaunch& p);
 cudaError_t dpso_begin(Instance& I, const DpsoLaunch& p, void* ws, cudaStream_t s);
 // iterations t0..t1-1 of Alg. 2 (one kernel launch each)

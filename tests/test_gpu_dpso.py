@@ -170,3 +170,24 @@ def test_config4_full_size_parity(lib):
     assert (got[0], got[2]) == (ref["E_best"], ref["id"])
     assert np.array_equal(got[1], ref["best"])
     assert np.array_equal(sw.trace.cpu().numpy(), ref["gbest_trace"])
+
+
+@pytest.mark.parametrize("kernel", ["warp", "group"])
+@pytest.mark.parametrize("n,particles,iters,problem", [(37, 100, 25, "cdd"), (300, 64, 10, "ucddcp"),
+                                                      (1000, 40, 6, "cdd")])
+def test_dpso_both_kernels(lib, monkeypatch, kernel, n, particles, iters, problem):
+    # the warp-per-particle and the group-layout iteration kernels are both bit-exact (the library
+    # picks by n; CDD_DPSO forces one)
+    import torch
+
+    monkeypatch.setenv("CDD_DPSO", kernel)
+    inst = gen.ucddcp_instance(n, 5) if problem == "ucddcp" else gen.cdd_instance(n, 4, 0.4)
+    ins = lib.Instance.from_gen(inst)
+    res = lib.dpso_run(ins, particles, iters, problem=problem, seed=77 + n, trace=True)
+    torch.cuda.synchronize()
+    pen, perm, gid = lib.best_get(ins)
+    P = oracle.CDD if problem == "cdd" else oracle.UCDDCP
+    ref = oracle.dpso_run(oracle.Problem.from_instance(inst),
+                          oracle.dpso_params(problem=P, particles=particles, iters=iters, seed=77 + n), trace=True)
+    assert np.array_equal(res["gbest_trace"].cpu().numpy()[:iters], ref["gbest_trace"])
+    assert (pen, gid) == (ref["E_best"], ref["id"]) and np.array_equal(perm, ref["best"])
