@@ -78,6 +78,8 @@ typedef struct cdd_instance cdd_instance; /* opaque, library-owned, bound to one
  *              255, the packed UCDDCP record fits 32 bits): packed 8/16-bit job records, int32
  *              arithmetic, the tuned kernels (every Biskup-Feldmann instance, p <= 20, alpha <= 10,
  *              beta <= 15, at n <= 1000).  The group SA kernels also need alpha, beta <= 255.
+ *              An instance whose CDD data fit but whose UCDDCP record does not runs the CDD on the
+ *              fast path and the UCDDCP on the generic one.
  *   generic -- everything else: int32 fields per job, int64 arithmetic, a warp (n <= 2048) or a
  *              CTA per sequence.  Serves the batched evaluators, the schedules, asynchronous SA
  *              (every move) and T0; synchronous SA and DPSO return CDD_EINVAL; the best result is
@@ -89,8 +91,9 @@ CDD_API int cdd_instance_create(int32_t n, const int32_t *p, const int32_t *alph
                         const int32_t *m, const int32_t *gamma, int64_t d, int device,
                         cdd_instance **out);
 CDD_API int cdd_instance_destroy(cdd_instance *inst);
-/* n, d, sum of p, and flags (bit0: UCDDCP data present, bit1: d >= sum p, bit2: generic path).
- * Any out may be NULL. */
+/* n, d, sum of p, and flags (bit0: UCDDCP data present, bit1: d >= sum p, bit2: the CDD runs on
+ * the generic path, bit3: the UCDDCP runs on the generic path -- its packed record does not fit
+ * even where the CDD's does).  Any out may be NULL. */
 CDD_API int cdd_instance_query(const cdd_instance *inst, int32_t *n, int64_t *d, int64_t *sum_p,
                        int32_t *flags);
 

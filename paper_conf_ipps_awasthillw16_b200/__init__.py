@@ -155,7 +155,8 @@ class Instance:
         n, d, sp, fl = C.c_int32(), C.c_int64(), C.c_int64(), C.c_int32()
         _check(_lib.cdd_instance_query(self.handle, C.byref(n), C.byref(d), C.byref(sp), C.byref(fl)))
         return dict(n=n.value, d=d.value, sum_p=sp.value, has_ucddcp=bool(fl.value & 1),
-                    unrestricted=bool(fl.value & 2), generic=bool(fl.value & 4))
+                    unrestricted=bool(fl.value & 2), generic=bool(fl.value & 4),
+                    ucddcp_generic=bool(fl.value & 8))
 
     @property
     def handle(self):

@@ -193,16 +193,17 @@ int cdd_instance_create(int32_t n, const int32_t* p, const int32_t* alpha, const
     // p, M, P-M bytes, alpha, beta, gamma 16-bit halves) and int32 penalties
     const int wp = bits_for(32ull * (uint64_t)pmax), wa = bits_for(32ull * (uint64_t)amax),
               wb = bits_for(32ull * (uint64_t)bmax);
-    bool packed = n <= 1024 && sa < 65536 && sb < 65536 && (sa + sb) * sp < (int64_t)INT32_MAX &&
-                  wp + wa + wb <= 32 && pmax <= 255 && 32 * amax < 65536 && 32 * bmax < 65536;
+    const bool packed = n <= 1024 && sa < 65536 && sb < 65536 && (sa + sb) * sp < (int64_t)INT32_MAX &&
+                        wp + wa + wb <= 32 && pmax <= 255 && 32 * amax < 65536 && 32 * bmax < 65536;
     int ua = 0, ub = 0, um = 0, ux = 0, ug = 0;
+    bool ucd_packed = false;
     if (m) {
         ua = bits_for(32ull * (uint64_t)amax);
         ub = bits_for(32ull * (uint64_t)bmax);
         um = bits_for((uint64_t)mmax);
         ux = bits_for((uint64_t)xmax);
         ug = bits_for((uint64_t)gmax);
-        packed = packed && gmax < 65536 && xmax <= 255 && ua + ub + um + ux + ug <= 32;
+        ucd_packed = packed && gmax < 65536 && xmax <= 255 && ua + ub + um + ux + ug <= 32;
     }
     auto* I = new cdd_instance();
     I->device = device;
@@ -228,14 +229,19 @@ int cdd_instance_create(int32_t n, const int32_t* p, const int32_t* alpha, const
         free_instance(I);
         return cuda_fail(e, "cdd_instance_create");
     }
-    if (!packed) {
-        I->wide = true;
-        I->has_ucd = m != nullptr;
+    // the generic tables serve the CDD when the packed records do not fit, the UCDDCP when its own
+    // packed record does not (the CDD side of such an instance stays on the fast path)
+    I->has_ucd = m != nullptr;
+    I->wide = !packed;
+    I->ucd_wide = m != nullptr && !ucd_packed;
+    if (I->wide || I->ucd_wide) {
         const int rc = create_wide(I, n, p, alpha, beta, m, gamma);
         if (rc != CDD_OK) {
             free_instance(I);
             return rc;
         }
+    }
+    if (!packed) {
         *out = I;
         return CDD_OK;
     }
@@ -247,8 +253,7 @@ int cdd_instance_create(int32_t n, const int32_t* p, const int32_t* alpha, const
     std::vector<uint32_t> rc(n), ru;
     for (int i = 0; i < n; ++i)
         rc[i] = (uint32_t)p[i] | ((uint32_t)alpha[i] << I->lay_cdd.sa) | ((uint32_t)beta[i] << I->lay_cdd.sb);
-    if (m) {
-        I->has_ucd = true;
+    if (ucd_packed) {
         auto& L = I->lay_ucd;
         L.amask = mask_of(ua);
         L.sb = ua;
@@ -264,14 +269,14 @@ int cdd_instance_create(int32_t n, const int32_t* p, const int32_t* alpha, const
                     ((uint32_t)(p[i] - m[i]) << L.sx) | ((uint32_t)gamma[i] << L.sg);
     }
     chk(cudaMalloc(&I->rec_cdd, sizeof(uint32_t) * n));
-    if (I->has_ucd) chk(cudaMalloc(&I->rec_ucd, sizeof(uint32_t) * n));
+    if (ucd_packed) chk(cudaMalloc(&I->rec_ucd, sizeof(uint32_t) * n));
     std::vector<uint32_t> tab(n);
     std::vector<uint8_t> tp(n), tm(n), tx(n);
     std::vector<uint16_t> tg(n);
     for (int i = 0; i < n; ++i) {
         tab[i] = (uint32_t)alpha[i] | ((uint32_t)beta[i] << 16);
         tp[i] = (uint8_t)p[i];
-        if (m) {
+        if (ucd_packed) {
             tm[i] = (uint8_t)m[i];
             tx[i] = (uint8_t)(p[i] - m[i]);
             tg[i] = (uint16_t)gamma[i];
@@ -280,12 +285,13 @@ int cdd_instance_create(int32_t n, const int32_t* p, const int32_t* alpha, const
     chk(cudaMalloc(&I->tab_ab, sizeof(uint32_t) * n));
     chk(cudaMalloc(&I->tab_p, n));
     I->ab16_ok = amax <= 255 && bmax <= 255;
+    I->ab85_ok = amax <= 85 && bmax <= 85;
     std::vector<uint16_t> tab16(n);
     for (int i = 0; i < n; ++i) tab16[i] = (uint16_t)((alpha[i] & 0xff) | ((beta[i] & 0xff) << 8));
     chk(cudaMalloc(&I->tab_ab16, sizeof(uint16_t) * n));
     if (e == cudaSuccess)
         chk(cudaMemcpy(I->tab_ab16, tab16.data(), sizeof(uint16_t) * n, cudaMemcpyHostToDevice));
-    if (I->has_ucd) {
+    if (ucd_packed) {
         chk(cudaMalloc(&I->tab_m, n));
         chk(cudaMalloc(&I->tab_x, n));
         chk(cudaMalloc(&I->tab_g, sizeof(uint16_t) * n));
@@ -293,7 +299,7 @@ int cdd_instance_create(int32_t n, const int32_t* p, const int32_t* alpha, const
     if (e == cudaSuccess) {
         chk(cudaMemcpy(I->tab_ab, tab.data(), sizeof(uint32_t) * n, cudaMemcpyHostToDevice));
         chk(cudaMemcpy(I->tab_p, tp.data(), n, cudaMemcpyHostToDevice));
-        if (I->has_ucd) {
+        if (ucd_packed) {
             chk(cudaMemcpy(I->tab_m, tm.data(), n, cudaMemcpyHostToDevice));
             chk(cudaMemcpy(I->tab_x, tx.data(), n, cudaMemcpyHostToDevice));
             chk(cudaMemcpy(I->tab_g, tg.data(), sizeof(uint16_t) * n, cudaMemcpyHostToDevice));
@@ -301,7 +307,7 @@ int cdd_instance_create(int32_t n, const int32_t* p, const int32_t* alpha, const
     }
     if (e == cudaSuccess) {
         chk(cudaMemcpy(I->rec_cdd, rc.data(), sizeof(uint32_t) * n, cudaMemcpyHostToDevice));
-        if (I->has_ucd) chk(cudaMemcpy(I->rec_ucd, ru.data(), sizeof(uint32_t) * n, cudaMemcpyHostToDevice));
+        if (ucd_packed) chk(cudaMemcpy(I->rec_ucd, ru.data(), sizeof(uint32_t) * n, cudaMemcpyHostToDevice));
         chk(cdd::probe_smem_base(&I->smem_base));
     }
     if (e != cudaSuccess) {
@@ -323,7 +329,7 @@ int cdd_instance_query(const cdd_instance* I, int32_t* n, int64_t* d, int64_t* s
     if (n) *n = I->n;
     if (d) *d = I->d;
     if (sum_p) *sum_p = I->sum_p;
-    if (flags) *flags = (I->has_ucd ? 1 : 0) | (I->d >= I->sum_p ? 2 : 0) | (I->wide ? 4 : 0);
+    if (flags) *flags = (I->has_ucd ? 1 : 0) | (I->d >= I->sum_p ? 2 : 0) | (I->wide ? 4 : 0) | (I->ucd_wide ? 8 : 0);
     return CDD_OK;
 }
 
@@ -337,10 +343,13 @@ static int check_batch_args(const cdd_instance* I, const int16_t* perms, int64_t
 }
 
 // fast (packed) or generic (wide) evaluator
+// the generic kernels serve this problem on this instance
+static bool generic(const cdd_instance& I, bool ucd) { return ucd ? I.ucd_wide : I.wide; }
+
 static cudaError_t any_eval(const cdd_instance& I, bool ucd, const int16_t* perms, int64_t ld, int64_t batch,
                             int64_t* out, cudaStream_t s) {
-    return I.wide ? cdd::launch_wide_eval(I, ucd, perms, ld, batch, out, s)
-                  : cdd::launch_eval_batch(I, ucd, perms, ld, batch, out, s);
+    return generic(I, ucd) ? cdd::launch_wide_eval(I, ucd, perms, ld, batch, out, s)
+                           : cdd::launch_eval_batch(I, ucd, perms, ld, batch, out, s);
 }
 
 static int eval_common(cdd_instance* I, bool ucd, const int16_t* perms, int64_t ld, int64_t batch,
@@ -374,7 +383,7 @@ int cdd_schedule_batch(cdd_instance* I, cdd_problem problem, const int16_t* perm
     if (batch > 0 && (!C || !start || (ucd && !X))) return fail(CDD_EINVAL, "C/start (and X for UCDDCP) must be non-NULL");
     if (ucd && (!I->has_ucd || I->d < I->sum_p)) return fail(CDD_EINVAL, "instance not usable for UCDDCP (no m/gamma, or d < sum p)");
     DeviceGuard g(I->device);
-    cudaError_t e = I->wide ? cdd::launch_wide_schedule(*I, ucd, perms, ld, batch, C, X, start, penalty, as_stream(stream))
+    cudaError_t e = generic(*I, ucd) ? cdd::launch_wide_schedule(*I, ucd, perms, ld, batch, C, X, start, penalty, as_stream(stream))
                             : cdd::launch_schedule(*I, ucd, perms, ld, batch, C, X, start, penalty, as_stream(stream));
     return e == cudaSuccess ? CDD_OK : cuda_fail(e, "cdd_schedule_batch");
 }
@@ -447,9 +456,9 @@ static int sa_validate(const cdd_instance* I, const sa_params* p, cdd::SaLaunch*
     if (std::isnan(p->T0)) return fail(CDD_EINVAL, "T0 is NaN");
     if (p->lanes != 0 && p->lanes != 4 && p->lanes != 8 && p->lanes != 16 && p->lanes != 32)
         return fail(CDD_EINVAL, "lanes must be 0, 4, 8, 16 or 32");
-    if (p->lanes >= 4 && p->lanes <= 16 && !I->ab16_ok)
-        return fail(CDD_EINVAL, "lanes 4/8/16 need alpha, beta <= 255 (16-bit records, fast path)");
-    if (I->wide && !(p->T0 > 0) && !p->T0_in &&
+    if (p->lanes >= 4 && p->lanes <= 16 && (!I->ab16_ok || generic(*I, ucd)))
+        return fail(CDD_EINVAL, "lanes 4/8/16 need the fast path with alpha, beta <= 255 (16-bit records)");
+    if (generic(*I, ucd) && !(p->T0 > 0) && !p->T0_in &&
         (unsigned __int128)p->t0_samples * (unsigned __int128)(uint64_t)I->penalty_bound >= ((unsigned __int128)1 << 65))
         return fail(CDD_EINVAL, "T0 from samples: t0_samples * penalty bound must be < 2^65 (exact 128-bit moments); give T0");
     if (p->lanes == 4 && I->n > 256) return fail(CDD_EINVAL, "lanes = 4 supports n <= 256");
@@ -479,7 +488,7 @@ size_t sa_workspace_size(const cdd_instance* I, const sa_params* p) {
     cdd::SaLaunch L{};
     if (sa_validate(I, p, &L) != CDD_OK) return 0;
     DeviceGuard g(I->device);
-    return I->wide ? cdd::wide_sa_workspace_bytes(*I, L) : cdd::sa_workspace_bytes(*I, L);
+    return generic(*I, L.ucd) ? cdd::wide_sa_workspace_bytes(*I, L) : cdd::sa_workspace_bytes(*I, L);
 }
 
 static int sync_validate(const cdd_instance* I, const sa_sync_params* q, cdd::SaLaunch* L) {
@@ -489,7 +498,8 @@ static int sync_validate(const cdd_instance* I, const sa_sync_params* q, cdd::Sa
         return fail(CDD_EINVAL, "levels * markov_len must be < 2^32");
     if (q->lanes != 0 && q->lanes != 4 && q->lanes != 8 && q->lanes != 16)
         return fail(CDD_EINVAL, "synchronous SA runs on lanes 0, 4, 8 or 16");
-    if (!I->ab16_ok) return fail(CDD_EINVAL, "synchronous SA needs the fast path (packed records, alpha, beta <= 255)");
+    if (!I->ab16_ok || generic(*I, q->problem == CDD_PROBLEM_UCDDCP))
+        return fail(CDD_EINVAL, "synchronous SA needs the fast path (packed records, alpha, beta <= 255)");
     sa_params p{};
     p.problem = q->problem;
     p.chains = q->chains;
@@ -591,10 +601,11 @@ int sa_run(cdd_instance* I, const sa_params* p, void* ws, size_t ws_bytes, void*
     int rc = sa_validate(I, p, &L);
     if (rc != CDD_OK) return rc;
     DeviceGuard g(I->device);
-    const size_t need = I->wide ? cdd::wide_sa_workspace_bytes(*I, L) : cdd::sa_workspace_bytes(*I, L);
+    const size_t need = generic(*I, L.ucd) ? cdd::wide_sa_workspace_bytes(*I, L) : cdd::sa_workspace_bytes(*I, L);
     if (!ws || ws_bytes < need)
         return fail(CDD_ENOMEM, "workspace too small: need " + std::to_string(need) + " bytes");
-    cudaError_t e = I->wide ? cdd::launch_wide_sa(*I, L, ws, as_stream(stream)) : cdd::launch_sa(*I, L, ws, as_stream(stream));
+    cudaError_t e = generic(*I, L.ucd) ? cdd::launch_wide_sa(*I, L, ws, as_stream(stream))
+                                       : cdd::launch_sa(*I, L, ws, as_stream(stream));
     if (e != cudaSuccess) return cuda_fail(e, "sa_run");
     I->has_best = true;
     return CDD_OK;
@@ -616,10 +627,10 @@ int sa_t0(cdd_instance* I, cdd_problem problem, uint64_t seed, int64_t samples, 
     int rc = sa_validate(I, &p, &L);
     if (rc != CDD_OK) return rc;
     DeviceGuard g(I->device);
-    const size_t need = I->wide ? cdd::wide_sa_workspace_bytes(*I, L) : cdd::sa_workspace_bytes(*I, L);
+    const size_t need = generic(*I, L.ucd) ? cdd::wide_sa_workspace_bytes(*I, L) : cdd::sa_workspace_bytes(*I, L);
     if (!ws || ws_bytes < need)
         return fail(CDD_ENOMEM, "workspace too small: need " + std::to_string(need) + " bytes");
-    cudaError_t e = I->wide ? cdd::launch_wide_t0(*I, L.ucd, seed, samples, T0_dev, ws, as_stream(stream))
+    cudaError_t e = generic(*I, L.ucd) ? cdd::launch_wide_t0(*I, L.ucd, seed, samples, T0_dev, ws, as_stream(stream))
                             : cdd::launch_t0(*I, L.ucd, seed, samples, T0_dev, ws, as_stream(stream));
     return e == cudaSuccess ? CDD_OK : cuda_fail(e, "sa_t0");
 }
@@ -630,7 +641,7 @@ static int dpso_validate(const cdd_instance* I, const dpso_params* p, cdd::DpsoL
     const bool ucd = p->problem == CDD_PROBLEM_UCDDCP;
     if (ucd && (!I->has_ucd || I->d < I->sum_p)) return fail(CDD_EINVAL, "instance not usable for UCDDCP (no m/gamma, or d < sum p)");
     if (I->n < 2) return fail(CDD_EINVAL, "DPSO needs n >= 2");
-    if (I->wide) return fail(CDD_EINVAL, "DPSO runs on the fast path only (packed records: n <= 1024, p <= 255, ...)");
+    if (generic(*I, ucd)) return fail(CDD_EINVAL, "DPSO runs on the fast path only (packed records: n <= 1024, p <= 255, ...)");
     if (p->particles < 1 || p->particles >= (1ll << 31)) return fail(CDD_EINVAL, "particles must be in [1, 2^31)");
     if (p->iters < 0 || p->iters >= (int64_t)UINT32_MAX) return fail(CDD_EINVAL, "iters must be in [0, 2^32)");
     if (p->particle_offset + (uint64_t)p->particles > (1ull << 32)) return fail(CDD_EINVAL, "particle ids must fit 32 bits");

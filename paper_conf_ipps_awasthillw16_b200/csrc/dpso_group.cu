@@ -51,6 +51,7 @@ struct DgArgs {
     unsigned long long* ctakeys;  // [gridDim]: each CTA's minimum key of the current publish
     int64_t* trace;
     int np;
+    bool quad;  // CDD with max(alpha, beta) <= 85 (the evaluator's quad pass)
     // tables by job id (global; staged in shared memory per CTA): CDD alpha|beta<<8 | p<<16;
     // UCDDCP alpha|beta<<8 | gamma<<16 and M | X<<8
     const uint16_t* ab16;
@@ -67,7 +68,6 @@ template <int DG, int E, bool UCD>
 struct DgSmem {
     using C = GChain<DG, E, UCD>;
     static constexpr int NP = C::NP;
-    static_assert(2 * NP <= C::AB_BYTES, "inv aliases the record area");
     static constexpr int GROUP = (C::BYTES + 4 * NP + 15) / 16 * 16;  // chain records, ids, inv
     static constexpr int IDS = C::BYTES, INV = C::BYTES + 2 * NP;
     static constexpr int TAB = UCD ? NP * 6 : NP * 4;
@@ -265,7 +265,6 @@ __device__ __forceinline__ uint2 dg_build(const GChain<DG, E, UCD>& ch, const ui
     constexpr int NP = C::NP;
     const uint32_t* t32 = reinterpret_cast<const uint32_t*>(tab);
     const uint16_t* t16 = reinterpret_cast<const uint16_t*>(tab + 4 * NP);
-    uint8_t* abr = reinterpret_cast<uint8_t*>(ch.ab()) + l * C::AS;
     uint8_t* pr = ch.pb() + l * C::PS;
     uint32_t tAB = 0, tP = 0;
 #pragma unroll 2
@@ -275,15 +274,16 @@ __device__ __forceinline__ uint2 dg_build(const GChain<DG, E, UCD>& ch, const ui
         uint32_t r[8];
 #pragma unroll
         for (int j = 0; j < 8; ++j) r[j] = t32[half16(q, j)];  // pads hold ids >= n: zero records
-        uint32_t w[4];
-#pragma unroll
-        for (int j = 0; j < 4; ++j) {
-            w[j] = __byte_perm(r[2 * j], r[2 * j + 1], 0x5410u);  // alpha|beta of two positions
-            tAB = __dp4a(w[j], 0x00010001u, tAB);
-            tAB += __dp4a(w[j], 0x01000100u, 0u) << 16;
-        }
-        *reinterpret_cast<uint4*>(abr + 2 * c) = make_uint4(w[0], w[1], w[2], w[3]);
         if constexpr (UCD) {
+            uint8_t* abr = reinterpret_cast<uint8_t*>(ch.ab()) + l * C::AS;
+            uint32_t w[4];
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+                w[j] = __byte_perm(r[2 * j], r[2 * j + 1], 0x5410u);  // alpha|beta of two positions
+                tAB = __dp4a(w[j], 0x00010001u, tAB);
+                tAB += __dp4a(w[j], 0x01000100u, 0u) << 16;
+            }
+            *reinterpret_cast<uint4*>(abr + 2 * c) = make_uint4(w[0], w[1], w[2], w[3]);
             uint32_t g2[4];
 #pragma unroll
             for (int j = 0; j < 4; ++j) g2[j] = __byte_perm(r[2 * j], r[2 * j + 1], 0x7632u);  // gamma pairs
@@ -301,9 +301,19 @@ __device__ __forceinline__ uint2 dg_build(const GChain<DG, E, UCD>& ch, const ui
             *reinterpret_cast<uint2*>(ch.xb() + l * C::PS + c) = make_uint2(x0, x1);
             tP = __dp4a(m0, 0x01010101u, __dp4a(m1, 0x01010101u, tP));
         } else {
-            const uint32_t p0 = __byte_perm(__byte_perm(r[0], r[1], 0x0062u), __byte_perm(r[2], r[3], 0x0062u), 0x5410u);
-            const uint32_t p1 = __byte_perm(__byte_perm(r[4], r[5], 0x0062u), __byte_perm(r[6], r[7], 0x0062u), 0x5410u);
+            // CDD byte rows: alpha (byte 0 of a record), beta (byte 1), P (byte 2)
+            auto quad = [&](int b, uint32_t sel) {
+                return __byte_perm(__byte_perm(r[b], r[b + 1], sel), __byte_perm(r[b + 2], r[b + 3], sel), 0x5410u);
+            };
+            const uint32_t a0 = quad(0, 0x0040u), a1 = quad(4, 0x0040u);
+            const uint32_t b0 = quad(0, 0x0051u), b1 = quad(4, 0x0051u);
+            const uint32_t p0 = quad(0, 0x0062u), p1 = quad(4, 0x0062u);
+            const int o = l * C::RS + c;
+            *reinterpret_cast<uint2*>(ch.a8() + o) = make_uint2(a0, a1);
+            *reinterpret_cast<uint2*>(ch.b8() + o) = make_uint2(b0, b1);
             *reinterpret_cast<uint2*>(pr + c) = make_uint2(p0, p1);
+            tAB += __dp4a(a0, 0x01010101u, __dp4a(a1, 0x01010101u, 0u)) |
+                   (__dp4a(b0, 0x01010101u, __dp4a(b1, 0x01010101u, 0u)) << 16);
             tP = __dp4a(p0, 0x01010101u, __dp4a(p1, 0x01010101u, tP));
         }
     }
@@ -312,11 +322,12 @@ __device__ __forceinline__ uint2 dg_build(const GChain<DG, E, UCD>& ch, const ui
 }
 
 template <int DG, int E, bool UCD>
-__device__ __forceinline__ int32_t dg_eval(const GChain<DG, E, UCD>& ch, int l, int gbase, int n, int32_t d, uint2 t) {
+__device__ __forceinline__ int32_t dg_eval(const GChain<DG, E, UCD>& ch, int l, int gbase, int n, int32_t d, uint2 t,
+                                          bool quad) {
     if constexpr (UCD)
         return gchain_eval_ucddcp<DG, E>(ch, l, gbase, n, t.x);
     else
-        return gchain_eval_cdd<DG, E>(ch, l, gbase, n, d, t.x, t.y);
+        return gchain_eval_cdd<DG, E>(ch, l, gbase, n, d, t.x, t.y, quad);
 }
 
 // row copies between global memory and the group's shared-memory arrays (16 bytes per lane-step)
@@ -347,7 +358,7 @@ __global__ void __launch_bounds__(DgSmem<DG, E, UCD>::THREADS) dpsog_init_kernel
     uint8_t* gb = smem + S::P_OFF + (size_t)(wib * (32 / DG) + grp) * S::GROUP;
     const C ch{gb};
     uint16_t* ids = reinterpret_cast<uint16_t*>(gb + C::BYTES);
-    uint16_t* inv = reinterpret_cast<uint16_t*>(ch.ab());
+    uint16_t* inv = reinterpret_cast<uint16_t*>(gb + S::INV);
     uint32_t* words = reinterpret_cast<uint32_t*>(ch.pb());  // Philox staging (P rows are free here)
     const int n = a.n;
     const int per_cta = (int)(blockDim.x >> 5) * (32 / DG);
@@ -388,7 +399,7 @@ __global__ void __launch_bounds__(DgSmem<DG, E, UCD>::THREADS) dpsog_init_kernel
         }
         __syncwarp();
         const uint2 t = dg_build<DG, E, UCD>(ch, ids, smem, n, l);
-        const int32_t z = dg_eval<DG, E, UCD>(ch, l, gbase, n, a.d, t);
+        const int32_t z = dg_eval<DG, E, UCD>(ch, l, gbase, n, a.d, t, a.quad);
         if (active && l == 0) a.zb[i] = z;
         const unsigned long long key = active ? ((unsigned long long)(uint32_t)z << 32) | (uint32_t)gid : ULLONG_MAX;
         wkey = key < wkey ? key : wkey;
@@ -587,7 +598,7 @@ __global__ void __launch_bounds__(DgSmem<DG, E, UCD>::THREADS, 1) dpsog_iter_ker
             __syncwarp();
             // line 7: evaluate
             const uint2 tt = dg_build<DG, E, UCD>(ch, ids, smem, n, l);
-            const int32_t z = dg_eval<DG, E, UCD>(ch, l, gbase, n, a.d, tt);
+            const int32_t z = dg_eval<DG, E, UCD>(ch, l, gbase, n, a.d, tt, a.quad);
             // line 4 (iteration t+1): personal best
             int32_t best = zb;
             if (active && z < zb) {
@@ -741,6 +752,7 @@ static DgArgs dg_args(const Instance& I, const DpsoLaunch& p, const DpsoWsPtrs& 
     }
     a.trace = p.gbest_trace;
     a.np = w.np;
+    a.quad = I.ab85_ok && !getenv("CDD_SA_NO_QUAD");
     a.ab16 = I.tab_ab16;
     a.p = I.tab_p;
     a.m = I.tab_m;

@@ -50,13 +50,15 @@ struct Instance {
     uint32_t* tab_ab = nullptr;
     uint16_t* tab_ab16 = nullptr;  // alpha | beta << 8 (only when both <= 255: ab16_ok)
     bool ab16_ok = false;
+    bool ab85_ok = false;  // max(alpha, beta) <= 85: the CDD evaluator's quad pass (sa_group.cuh)
     uint32_t smem_base = 1024;  // shared-window address of dynamic shared memory (probed at create)
     uint8_t* tab_p = nullptr;
     uint8_t* tab_m = nullptr;
     uint8_t* tab_x = nullptr;
     uint16_t* tab_g = nullptr;
     // generic ("wide") path (wide.cu): instances outside the packed record ranges
-    bool wide = false;
+    bool wide = false;      // the CDD uses the generic kernels
+    bool ucd_wide = false;  // the UCDDCP uses the generic kernels (its packed record does not fit)
     int64_t penalty_bound = 0;  // (sum a + sum b) * sum p + sum gamma * sum (P - M) (< 2^62)
     int4* tab_w0 = nullptr;  // {P, alpha, beta, gamma} by job id
     int2* tab_w1 = nullptr;  // {M, P - M} by job id (UCDDCP)

@@ -64,6 +64,63 @@ struct GChain {
     static __device__ __forceinline__ int gh_h(int k) { return (k / E) * (GS / 2) + (k % E); }
 };
 
+// CDD chain: three byte rows per lane -- alpha, beta, P -- so that four consecutive positions of
+// one field are one 32-bit word.  With max(alpha, beta) <= 85 the pass then handles a quad of
+// positions in five instructions (byte-wise prefixes by one IMAD, IDP.4A against the P quad);
+// larger weights use 16-bit prefix pairs as the UCDDCP layout does.  Lane rows are padded by 16
+// bytes (E >= 32) so the lane-contiguous LDS.128 of a group is bank-conflict free.
+template <int G, int E>
+struct GChain<G, E, false> {
+    static constexpr int NP = G * E;
+    static constexpr int RS = E >= 32 ? E + 16 : E;  // bytes per lane row (each field)
+    static constexpr int PS = RS;
+    static constexpr int SPR = E >= G ? E / G : 1;   // boundary elements per lane
+    static constexpr int ROW_BYTES = (G * RS + 15) / 16 * 16;
+    static constexpr int OFF_B = ROW_BYTES, OFF_P = 2 * ROW_BYTES, OFF_T = 3 * ROW_BYTES;
+    static constexpr int BYTES = (OFF_T + G * 8 + 15) / 16 * 16;
+    static_assert(2 * NP + 16 * G <= BYTES, "FY staging (ids + Philox words) must fit");
+    uint8_t* base;
+    __device__ __forceinline__ uint8_t* a8() const { return base; }
+    __device__ __forceinline__ uint8_t* b8() const { return base + OFF_B; }
+    __device__ __forceinline__ uint8_t* pb() const { return base + OFF_P; }
+    __device__ __forceinline__ uint2* tot() const { return reinterpret_cast<uint2*>(base + OFF_T); }
+    static __device__ __forceinline__ int rb(int k) { return (k / E) * RS + (k % E); }
+    static __device__ __forceinline__ int pb_b(int k) { return rb(k); }
+};
+
+// N alpha bytes and N beta bytes (N >= 2, a multiple of 2) as N/2 words alpha|beta<<8 per
+// position, two positions per word (the 16-bit record pairs of the UCDDCP layout)
+template <int N>
+__device__ __forceinline__ void ab_pairs(const uint8_t* ar, const uint8_t* br, uint32_t (&w)[N / 2]) {
+    if constexpr (N >= 4) {
+        uint32_t a[N / 4], b[N / 4];
+        if constexpr (N >= 16) {
+#pragma unroll
+            for (int q = 0; q < N / 16; ++q) {
+                const uint4 x = *reinterpret_cast<const uint4*>(ar + 16 * q);
+                const uint4 y = *reinterpret_cast<const uint4*>(br + 16 * q);
+                a[4 * q] = x.x; a[4 * q + 1] = x.y; a[4 * q + 2] = x.z; a[4 * q + 3] = x.w;
+                b[4 * q] = y.x; b[4 * q + 1] = y.y; b[4 * q + 2] = y.z; b[4 * q + 3] = y.w;
+            }
+        } else if constexpr (N == 8) {
+            const uint2 x = *reinterpret_cast<const uint2*>(ar);
+            const uint2 y = *reinterpret_cast<const uint2*>(br);
+            a[0] = x.x; a[1] = x.y; b[0] = y.x; b[1] = y.y;
+        } else {
+            a[0] = *reinterpret_cast<const uint32_t*>(ar);
+            b[0] = *reinterpret_cast<const uint32_t*>(br);
+        }
+#pragma unroll
+        for (int q = 0; q < N / 4; ++q) {
+            w[2 * q] = __byte_perm(a[q], b[q], 0x5140u);
+            w[2 * q + 1] = __byte_perm(a[q], b[q], 0x7362u);
+        }
+    } else {
+        const uint32_t a = *reinterpret_cast<const uint16_t*>(ar), b = *reinterpret_cast<const uint16_t*>(br);
+        w[0] = __byte_perm(a, b, 0x5140u);
+    }
+}
+
 // alpha | beta << 8 (u16) -> alpha | beta << 16
 __device__ __forceinline__ uint32_t ab_wide(uint32_t r16) { return __byte_perm(r16, 0u, 0x4140u); }
 
@@ -115,7 +172,26 @@ __device__ __forceinline__ void load_b8(const uint8_t* row, uint32_t (&w)[E / 4]
     }
 }
 
-// SPR consecutive records of unit (lane row) `ls` starting at element e0, widened
+// SPR consecutive records of unit (lane row) `ls` starting at element e0, widened to alpha | beta << 16
+// (CDD byte rows)
+template <int SPR, int G, int E>
+__device__ __forceinline__ void load_spread(const GChain<G, E, false>& ch, int ls, int e0, bool in,
+                                            uint32_t (&rv)[SPR]) {
+    using C = GChain<G, E, false>;
+    const int o = ls * C::RS + e0;
+    if constexpr (SPR >= 2) {
+        uint32_t w[SPR / 2];
+        ab_pairs<SPR>(ch.a8() + o, ch.b8() + o, w);
+#pragma unroll
+        for (int i = 0; i < SPR / 2; ++i) {
+            rv[2 * i] = ab_wide(w[i] & 0xffffu);
+            rv[2 * i + 1] = ab_wide(w[i] >> 16);
+        }
+    } else {
+        rv[0] = in ? ((uint32_t)ch.a8()[o] | ((uint32_t)ch.b8()[o] << 16)) : 0u;
+    }
+}
+
 template <int SPR, class C>
 __device__ __forceinline__ void load_spread(const C& ch, int ls, int e0, bool in, uint32_t (&rv)[SPR]) {
     const uint16_t* src = ch.ab() + ls * (C::AS / 2) + e0;
@@ -160,11 +236,12 @@ __device__ __forceinline__ int32_t boundary_two_level(const GChain<G, E>& ch, in
     constexpr int SB = E / G;   // positions per sub-block (16 for E = 128, G = 8)
     constexpr int L2 = SB / G;  // positions per lane in level 2
     static_assert(SB % 8 == 0 && L2 >= 1 && L2 <= 4, "two-level boundary layout");
-    const uint8_t* arow = reinterpret_cast<const uint8_t*>(ch.ab()) + Ls * C::AS;
-    const uint8_t* prow = ch.pb() + Ls * C::PS;
+    const uint8_t* arow = ch.a8() + Ls * C::RS;
+    const uint8_t* brow = ch.b8() + Ls * C::RS;
+    const uint8_t* prow = ch.pb() + Ls * C::RS;
     // ---- level 1
     uint32_t w[SB / 2], q[SB / 4];
-    load_ab16<SB>(arow + 2 * SB * l, w);
+    ab_pairs<SB>(arow + SB * l, brow + SB * l, w);
     load_b8<SB>(prow + SB * l, q);
     uint32_t Pb1 = 0, Sb1 = 0, sig2 = 0, dot = 0;
 #pragma unroll
@@ -188,15 +265,11 @@ __device__ __forceinline__ int32_t boundary_two_level(const GChain<G, E>& ch, in
     auto spread = [&](int blk, uint32_t (&v)[L2]) -> uint32_t {
         const int e = SB * blk + L2 * l;
         uint32_t a2[(L2 + 1) / 2], pp;
-        if constexpr (L2 == 4) {
-            const uint2 x = *reinterpret_cast<const uint2*>(arow + 2 * e);
-            a2[0] = x.x; a2[1] = x.y;
-            pp = *reinterpret_cast<const uint32_t*>(prow + e);
-        } else if constexpr (L2 == 2) {
-            a2[0] = *reinterpret_cast<const uint32_t*>(arow + 2 * e);
-            pp = *reinterpret_cast<const uint16_t*>(prow + e);
+        if constexpr (L2 >= 2) {
+            ab_pairs<L2>(arow + e, brow + e, a2);
+            pp = L2 == 4 ? *reinterpret_cast<const uint32_t*>(prow + e) : (uint32_t)*reinterpret_cast<const uint16_t*>(prow + e);
         } else {
-            a2[0] = *reinterpret_cast<const uint16_t*>(arow + 2 * e);
+            a2[0] = (uint32_t)arow[e] | ((uint32_t)brow[e] << 8);
             pp = prow[e];
         }
         uint32_t tot = 0;
@@ -236,18 +309,12 @@ __device__ __forceinline__ int32_t boundary_two_level(const GChain<G, E>& ch, in
 }
 
 // CDD penalty of the group's chain.  tAB / tP: this lane's totals (maintained incrementally).
+// quad: max(alpha, beta) <= 85 (the byte-wise prefix of three weights never carries).
 template <int G, int E>
 __device__ __forceinline__ int32_t gchain_eval_cdd(const GChain<G, E>& ch, int l, int gbase, int n,
-                                                   int32_t d, uint32_t tAB, uint32_t tP) {
+                                                   int32_t d, uint32_t tAB, uint32_t tP, bool quad) {
     using C = GChain<G, E>;
     constexpr int SPR = C::SPR;
-#if CDD_SAG_PREFETCH
-    // pass-2 operands are loaded first so their latency hides behind the scans and the spread
-    uint32_t rr[E / 2];
-    uint32_t pw[E / 4];
-    load_ab16<E>(reinterpret_cast<const uint8_t*>(ch.ab()) + l * C::AS, rr);
-    load_b8<E>(ch.pb() + l * C::PS, pw);
-#endif
     const uint32_t iP = gscan<G>(tP);
     const uint32_t iAB = gscan<G>(tAB);
     const int32_t Pb = (int32_t)(iP - tP);
@@ -279,7 +346,7 @@ __device__ __forceinline__ int32_t gchain_eval_cdd(const GChain<G, E>& ch, int l
         load_spread<SPR>(ch, Ls, e0, lane_in, rv);
         constexpr int PW = SPR >= 4 ? SPR / 4 : 1;
         uint32_t pv[PW];
-        const uint8_t* psrc = ch.pb() + Ls * C::PS + e0;
+        const uint8_t* psrc = ch.pb() + Ls * C::RS + e0;
         if constexpr (SPR >= 16) {
 #pragma unroll
             for (int q = 0; q < SPR / 16; ++q) {
@@ -325,66 +392,46 @@ __device__ __forceinline__ int32_t gchain_eval_cdd(const GChain<G, E>& ch, int l
         corr = boundary_two_level<G, E>(ch, l, gbase, Ls, Lk, d, PbS, thr, key);
     }
 
-    // ---- F(C_{m'}): per pair, f2 = (s, s + x0) by PRMT + IMAD, IDP.2A with the pair of p bytes,
-    // s advanced by IDP.4A (x = alpha in early lanes, beta in tardy lanes)
+    // ---- F(C_{m'}) = sum_j p_j * (exclusive prefix of x within the lane row), x = alpha in early
+    // lanes, beta in tardy lanes
     const bool amode = l < Ls;
-    const uint32_t psel = amode ? 0x4044u : 0x4144u;
-    const uint32_t wsum = amode ? 0x00010001u : 0x01000100u;
-    uint32_t s = 0, acc = 0;
-#if CDD_SAG_PREFETCH
-#pragma unroll
-    for (int j = 0; j < E / 2; ++j) {
-        const uint32_t f2 = s * 0x10001u + __byte_perm(rr[j], 0u, psel);
-        acc = (j & 1) ? __dp2a_hi(f2, pw[j >> 1], acc) : __dp2a_lo(f2, pw[j >> 1], acc);
-        s = __dp4a(rr[j], wsum, s);
-    }
-#else
-    const uint8_t* arow = reinterpret_cast<const uint8_t*>(ch.ab()) + l * C::AS;
-    const uint8_t* prow = ch.pb() + l * C::PS;
+    const uint8_t* xrow = (amode ? ch.a8() : ch.b8()) + l * C::RS;
+    const uint8_t* prow = ch.pb() + l * C::RS;
     constexpr int CH = E >= 16 ? 16 : E;  // positions per chunk
-#if CDD_SAG_SPLITPASS
-    if constexpr (E >= 2 * CH) {
-        // two independent halves (ILP 2 on the s / acc dependency chains): the second half starts
-        // from s = 0 and is corrected by s_mid * (sum of p over the second half)
-        constexpr int HALF = E / 2;
-        uint32_t s2 = 0, acc2 = 0, p2 = 0;
-#pragma unroll
-        for (int c0 = 0; c0 < HALF; c0 += CH) {
-            uint32_t r[CH / 2], q[CH / 4], rb[CH / 2], qb[CH / 4];
-            load_ab16<CH>(arow + 2 * c0, r);
-            load_b8<CH>(prow + c0, q);
-            load_ab16<CH>(arow + 2 * (c0 + HALF), rb);
-            load_b8<CH>(prow + c0 + HALF, qb);
-#pragma unroll
-            for (int j = 0; j < CH / 2; ++j) {
-                const uint32_t f2 = s * 0x10001u + __byte_perm(r[j], 0u, psel);
-                const uint32_t g2 = s2 * 0x10001u + __byte_perm(rb[j], 0u, psel);
-                acc = (j & 1) ? __dp2a_hi(f2, q[j >> 1], acc) : __dp2a_lo(f2, q[j >> 1], acc);
-                acc2 = (j & 1) ? __dp2a_hi(g2, qb[j >> 1], acc2) : __dp2a_lo(g2, qb[j >> 1], acc2);
-                s = __dp4a(r[j], wsum, s);
-                s2 = __dp4a(rb[j], wsum, s2);
-            }
-#pragma unroll
-            for (int j = 0; j < CH / 4; ++j) p2 = __dp4a(qb[j], 0x01010101u, p2);
-        }
-        acc += acc2 + s * p2;
-    } else
-#endif
-    {
+    uint32_t s = 0, acc = 0;
+    if (quad) {
+        // per quad: byte-wise exclusive prefixes [0, x0, x0+x1, x0+x1+x2] by one IMAD, their dot
+        // with the P quad by IDP.4A, plus s * (sum of the P quad)
 #pragma unroll
         for (int c0 = 0; c0 < E; c0 += CH) {
-            uint32_t r[CH / 2], q[CH / 4];
-            load_ab16<CH>(arow + 2 * c0, r);
+            uint32_t x[CH / 4], q[CH / 4];
+            load_b8<CH>(xrow + c0, x);
             load_b8<CH>(prow + c0, q);
 #pragma unroll
-            for (int j = 0; j < CH / 2; ++j) {
-                const uint32_t f2 = s * 0x10001u + __byte_perm(r[j], 0u, psel);
-                acc = (j & 1) ? __dp2a_hi(f2, q[j >> 1], acc) : __dp2a_lo(f2, q[j >> 1], acc);
-                s = __dp4a(r[j], wsum, s);
+            for (int j = 0; j < CH / 4; ++j) {
+                acc = __dp4a(x[j] * 0x01010100u, q[j], acc);
+                acc += s * __dp4a(q[j], 0x01010101u, 0u);
+                s = __dp4a(x[j], 0x01010101u, s);
+            }
+        }
+    } else {
+        // pairs: f2 = (s, s + x_{2j}) in 16-bit halves, IDP.2A with the pair of p bytes
+#pragma unroll
+        for (int c0 = 0; c0 < E; c0 += CH) {
+            uint32_t x[CH / 4], q[CH / 4];
+            load_b8<CH>(xrow + c0, x);
+            load_b8<CH>(prow + c0, q);
+#pragma unroll
+            for (int j = 0; j < CH / 4; ++j) {
+                const uint32_t f0 = s * 0x10001u + __byte_perm(x[j], 0u, 0x4044u);
+                acc = __dp2a_lo(f0, q[j], acc);
+                s = __dp4a(x[j], 0x00000101u, s);
+                const uint32_t f1 = s * 0x10001u + __byte_perm(x[j], 0u, 0x4244u);
+                acc = __dp2a_hi(f1, q[j], acc);
+                s = __dp4a(x[j], 0x01010000u, s);
             }
         }
     }
-#endif
     const int32_t base = amode ? Ab : (Btot - Bb);
     const int32_t contrib = base * (int32_t)tP + (amode ? (int32_t)acc : -(int32_t)acc) + corr;
     return (int32_t)gsum<G>((uint32_t)contrib);

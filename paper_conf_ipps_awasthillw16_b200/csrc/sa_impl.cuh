@@ -210,6 +210,8 @@ struct SaGArgs {
     // quad-major space; chains split between two warps hand their state over through `hand`
     int64_t share;
     uint8_t* hand;
+    // CDD: max(alpha, beta) <= 85, the evaluator's quad pass applies (sa_group.cuh)
+    bool quad;
 };
 
 // State of one chain handed from the warp that ran its first steps to the warp finishing it.
@@ -225,6 +227,31 @@ __host__ __device__ constexpr size_t hand_warp_bytes(int np, int cpw) {
 // Alg. 1 line 1 for the group's chain: Fisher-Yates of the identity (ids staged in the AB area,
 // Philox words in batches of 4G behind them, swaps on the group's lane 0), ids to the global
 // current slot, then the records and the per-lane totals.
+// This lane's totals of its row: alpha | beta << 16 and P (UCDDCP: M).
+template <int G, int E, bool UCD>
+__device__ __forceinline__ uint2 gchain_lane_totals(const GChain<G, E, UCD>& ch, int l) {
+    using C = GChain<G, E, UCD>;
+    uint32_t tAB = 0, tP = 0;
+    if constexpr (UCD) {
+        for (int i = 0; i < E; ++i) {
+            tAB += ab_wide(ch.ab()[l * (C::AS / 2) + i]);
+            tP += ch.pb()[l * C::PS + i];
+        }
+    } else {
+        const uint8_t* ar = ch.a8() + l * C::RS;
+        const uint8_t* br = ch.b8() + l * C::RS;
+        const uint8_t* pr = ch.pb() + l * C::RS;
+        uint32_t ta = 0, tb = 0;
+        for (int i = 0; i < E; i += 4) {
+            ta = __dp4a(*reinterpret_cast<const uint32_t*>(ar + i), 0x01010101u, ta);
+            tb = __dp4a(*reinterpret_cast<const uint32_t*>(br + i), 0x01010101u, tb);
+            tP = __dp4a(*reinterpret_cast<const uint32_t*>(pr + i), 0x01010101u, tP);
+        }
+        tAB = ta | (tb << 16);
+    }
+    return make_uint2(tAB, tP);
+}
+
 template <int G, int E, bool UCD>
 __device__ void gchain_init(const GChain<G, E, UCD>& ch, int16_t* cur, int n, uint64_t seed,
                             uint64_t g, int l, const ChainTables& T, const int16_t* init, int* err,
@@ -232,8 +259,8 @@ __device__ void gchain_init(const GChain<G, E, UCD>& ch, int16_t* cur, int n, ui
     using C = GChain<G, E, UCD>;
     constexpr int NP = C::NP;
     // staging: NP ids then 4G Philox words, 2 NP + 16 G bytes <= C::BYTES (static_assert there)
-    uint16_t* ids = ch.ab();
-    uint32_t* words = reinterpret_cast<uint32_t*>(ch.ab() + NP);
+    uint16_t* ids = reinterpret_cast<uint16_t*>(ch.base);
+    uint32_t* words = reinterpret_cast<uint32_t*>(ids + NP);
     if (init)
         for (int k = l; k < NP; k += G) {
             uint32_t v = k < n ? (uint16_t)init[k] : 0u;
@@ -290,31 +317,30 @@ __device__ void gchain_init(const GChain<G, E, UCD>& ch, int16_t* cur, int n, ui
         for (int u = 0; u < 8; ++u) {
             const int k = k0 + u * G;
             const bool v = k < n;
-            ch.ab()[C::ab_h(k)] = v ? __ldg(T.ab16 + jj[u]) : (uint16_t)0;
+            const uint32_t ab = v ? __ldg(T.ab16 + jj[u]) : 0u;
             ch.pb()[C::pb_b(k)] = v ? __ldg(T.p + jj[u]) : (uint8_t)0;
             if constexpr (UCD) {
+                ch.ab()[C::ab_h(k)] = (uint16_t)ab;
                 ch.xb()[C::pb_b(k)] = v ? __ldg(T.x + jj[u]) : (uint8_t)0;
                 ch.gh()[C::gh_h(k)] = v ? __ldg(T.g + jj[u]) : (uint16_t)0;
+            } else {
+                ch.a8()[C::rb(k)] = (uint8_t)ab;
+                ch.b8()[C::rb(k)] = (uint8_t)(ab >> 8);
             }
         }
     }
     __syncwarp();
-    uint32_t tAB = 0, tP = 0;
-    for (int i = 0; i < E; ++i) {
-        tAB += ab_wide(ch.ab()[l * (C::AS / 2) + i]);
-        tP += ch.pb()[l * C::PS + i];
-    }
-    ch.tot()[l] = make_uint2(tAB, tP);
+    ch.tot()[l] = gchain_lane_totals(ch, l);
     __syncwarp();
 }
 
 template <int G, int E, bool UCD>
 __device__ __forceinline__ int32_t gchain_eval(const GChain<G, E, UCD>& ch, int l, int gbase, int n,
-                                               int32_t d, uint2 t) {
+                                               int32_t d, uint2 t, bool quad) {
     if constexpr (UCD)
         return gchain_eval_ucddcp<G, E>(ch, l, gbase, n, t.x);
     else
-        return gchain_eval_cdd<G, E>(ch, l, gbase, n, d, t.x, t.y);
+        return gchain_eval_cdd<G, E>(ch, l, gbase, n, d, t.x, t.y, quad);
 }
 
 // The data of one position, packed for shuffles: u0 = alpha|beta<<8 | P << 16 (CDD) or
@@ -327,7 +353,8 @@ __device__ __forceinline__ uint2 pos_read(const GChain<G, E, UCD>& ch, int k) {
         v.x = (uint32_t)ch.ab()[C::ab_h(k)] | ((uint32_t)ch.gh()[C::gh_h(k)] << 16);
         v.y = (uint32_t)ch.pb()[C::pb_b(k)] | ((uint32_t)ch.xb()[C::pb_b(k)] << 8);
     } else {
-        v.x = (uint32_t)ch.ab()[C::ab_h(k)] | ((uint32_t)ch.pb()[C::pb_b(k)] << 16);
+        const int i = C::rb(k);
+        v.x = (uint32_t)ch.a8()[i] | ((uint32_t)ch.b8()[i] << 8) | ((uint32_t)ch.pb()[i] << 16);
         v.y = 0;
     }
     return v;
@@ -336,13 +363,16 @@ __device__ __forceinline__ uint2 pos_read(const GChain<G, E, UCD>& ch, int k) {
 template <int G, int E, bool UCD>
 __device__ __forceinline__ void pos_write(const GChain<G, E, UCD>& ch, int k, uint2 v) {
     using C = GChain<G, E, UCD>;
-    ch.ab()[C::ab_h(k)] = (uint16_t)v.x;
     if constexpr (UCD) {
+        ch.ab()[C::ab_h(k)] = (uint16_t)v.x;
         ch.gh()[C::gh_h(k)] = (uint16_t)(v.x >> 16);
         ch.pb()[C::pb_b(k)] = (uint8_t)v.y;
         ch.xb()[C::pb_b(k)] = (uint8_t)(v.y >> 8);
     } else {
-        ch.pb()[C::pb_b(k)] = (uint8_t)(v.x >> 16);
+        const int i = C::rb(k);
+        ch.a8()[i] = (uint8_t)v.x;
+        ch.b8()[i] = (uint8_t)(v.x >> 8);
+        ch.pb()[i] = (uint8_t)(v.x >> 16);
     }
 }
 
@@ -407,8 +437,6 @@ template <int G, int E, bool UCD, bool IDS>
 __device__ __forceinline__ void group_rotate(const GChain<G, E, UCD>& ch, int16_t* ids, int lo, int hi,
                                              bool left, bool act, int l) {
     using C = GChain<G, E, UCD>;
-    uint8_t* abb = reinterpret_cast<uint8_t*>(ch.ab());
-    uint8_t* ghb = reinterpret_cast<uint8_t*>(ch.gh());
     const int c0 = lo & ~7, c1 = hi & ~7;
     const int nch = act && hi > lo ? (c1 - c0) / 8 + 1 : 0;
     const int rounds = (int)__reduce_max_sync(kFull, (uint32_t)((nch + G - 1) / G));
@@ -435,34 +463,47 @@ __device__ __forceinline__ void group_rotate(const GChain<G, E, UCD>& ch, int16_
                 A16 = *reinterpret_cast<const uint4*>(ids + c);
                 const uint32_t nb = nbv ? (uint32_t)(uint16_t)ids[kn] : 0u;
                 A16 = rot16(A16, nb, left, m8);
-            } else {
+            } else if constexpr (UCD) {
+                uint8_t* abb = reinterpret_cast<uint8_t*>(ch.ab());
+                uint8_t* ghb = reinterpret_cast<uint8_t*>(ch.gh());
                 A16 = *reinterpret_cast<const uint4*>(abb + 2 * C::ab_h(c));
                 P8 = *reinterpret_cast<const uint2*>(ch.pb() + C::pb_b(c));
                 const uint32_t nab = nbv ? (uint32_t)ch.ab()[C::ab_h(kn)] : 0u;
                 const uint32_t np8 = nbv ? (uint32_t)ch.pb()[C::pb_b(kn)] : 0u;
                 A16 = rot16(A16, nab, left, m8);
                 P8 = rot8(P8, np8, left, m8);
-                if constexpr (UCD) {
-                    G16 = *reinterpret_cast<const uint4*>(ghb + 2 * C::gh_h(c));
-                    X8 = *reinterpret_cast<const uint2*>(ch.xb() + C::pb_b(c));
-                    const uint32_t ng = nbv ? (uint32_t)ch.gh()[C::gh_h(kn)] : 0u;
-                    const uint32_t nx = nbv ? (uint32_t)ch.xb()[C::pb_b(kn)] : 0u;
-                    G16 = rot16(G16, ng, left, m8);
-                    X8 = rot8(X8, nx, left, m8);
-                }
+                G16 = *reinterpret_cast<const uint4*>(ghb + 2 * C::gh_h(c));
+                X8 = *reinterpret_cast<const uint2*>(ch.xb() + C::pb_b(c));
+                const uint32_t ng = nbv ? (uint32_t)ch.gh()[C::gh_h(kn)] : 0u;
+                const uint32_t nx = nbv ? (uint32_t)ch.xb()[C::pb_b(kn)] : 0u;
+                G16 = rot16(G16, ng, left, m8);
+                X8 = rot8(X8, nx, left, m8);
+            } else {
+                // CDD: the alpha, beta and P byte rows (A16.x/.y carry alpha, .z/.w beta)
+                const int i = C::rb(c), in = C::rb(kn);
+                const uint2 a8 = *reinterpret_cast<const uint2*>(ch.a8() + i);
+                const uint2 b8 = *reinterpret_cast<const uint2*>(ch.b8() + i);
+                P8 = *reinterpret_cast<const uint2*>(ch.pb() + i);
+                const uint2 ra = rot8(a8, nbv ? (uint32_t)ch.a8()[in] : 0u, left, m8);
+                const uint2 rbt = rot8(b8, nbv ? (uint32_t)ch.b8()[in] : 0u, left, m8);
+                A16 = make_uint4(ra.x, ra.y, rbt.x, rbt.y);
+                P8 = rot8(P8, nbv ? (uint32_t)ch.pb()[in] : 0u, left, m8);
             }
         }
         __syncwarp();
         if (v && m8) {
             if constexpr (IDS) {
                 *reinterpret_cast<uint4*>(ids + c) = A16;
-            } else {
-                *reinterpret_cast<uint4*>(abb + 2 * C::ab_h(c)) = A16;
+            } else if constexpr (UCD) {
+                *reinterpret_cast<uint4*>(reinterpret_cast<uint8_t*>(ch.ab()) + 2 * C::ab_h(c)) = A16;
                 *reinterpret_cast<uint2*>(ch.pb() + C::pb_b(c)) = P8;
-                if constexpr (UCD) {
-                    *reinterpret_cast<uint4*>(ghb + 2 * C::gh_h(c)) = G16;
-                    *reinterpret_cast<uint2*>(ch.xb() + C::pb_b(c)) = X8;
-                }
+                *reinterpret_cast<uint4*>(reinterpret_cast<uint8_t*>(ch.gh()) + 2 * C::gh_h(c)) = G16;
+                *reinterpret_cast<uint2*>(ch.xb() + C::pb_b(c)) = X8;
+            } else {
+                const int i = C::rb(c);
+                *reinterpret_cast<uint2*>(ch.a8() + i) = make_uint2(A16.x, A16.y);
+                *reinterpret_cast<uint2*>(ch.b8() + i) = make_uint2(A16.z, A16.w);
+                *reinterpret_cast<uint2*>(ch.pb() + i) = P8;
             }
         }
         __syncwarp();
@@ -561,7 +602,7 @@ __global__ void __launch_bounds__(kGThreads, sag_min_blocks<G, E, UCD>()) sa_gro
         double T;
         if (!restore) {
             tt = ch.tot()[l];
-            Ecur = gchain_eval<G, E, UCD>(ch, l, gbase, n, a.d, tt);
+            Ecur = gchain_eval<G, E, UCD>(ch, l, gbase, n, a.d, tt, a.quad);
             Ebest = Ecur;
             cur_is_best = true;
             T = T0;
@@ -596,7 +637,7 @@ __global__ void __launch_bounds__(kGThreads, sag_min_blocks<G, E, UCD>()) sa_gro
                 const uint2 tn = make_uint2(tt.x + dt.x, tt.y + dt.y);
                 ch.tot()[l] = tn;
                 __syncwarp();
-                const int32_t En = gchain_eval<G, E, UCD>(ch, l, gbase, n, a.d, tn);
+                const int32_t En = gchain_eval<G, E, UCD>(ch, l, gbase, n, a.d, tn, a.quad);
                 const int32_t delta = Ecur - En;
                 const bool acc = delta >= 0 || metropolis_accept(delta, T, uw);
                 if (TRACE && active && l == 0)
@@ -649,7 +690,7 @@ __global__ void __launch_bounds__(kGThreads, sag_min_blocks<G, E, UCD>()) sa_gro
             __syncwarp();
             const uint2 tn = ch.tot()[l];
             // line 6
-            const int32_t En = gchain_eval<G, E, UCD>(ch, l, gbase, n, a.d, tn);
+            const int32_t En = gchain_eval<G, E, UCD>(ch, l, gbase, n, a.d, tn, a.quad);
             // line 7
             const int32_t delta = Ecur - En;
             const bool acc = delta >= 0 || metropolis_accept(delta, T, uw);
@@ -764,7 +805,7 @@ __global__ void __launch_bounds__(kGThreads, sag_min_blocks<G, E, UCD>()) sa_gro
 // resident at once than with a warp per sample.  Same words (tag T0, id = sample) and the same
 // evaluator as the SA chains, so Z is bit-identical to t0_sample_kernel's.
 template <int G, int E, bool UCD>
-__global__ void __launch_bounds__(kGThreads) t0_group_kernel(ChainTables T, int n, int32_t d, uint64_t seed,
+__global__ void __launch_bounds__(kGThreads) t0_group_kernel(ChainTables T, int n, int32_t d, bool quad, uint64_t seed,
                                                             int64_t samples, int16_t* scratch, int64_t* Z) {
     using C = GChain<G, E, UCD>;
     constexpr int CPW = 32 / G;
@@ -779,7 +820,7 @@ __global__ void __launch_bounds__(kGThreads) t0_group_kernel(ChainTables T, int 
         // (groups past the last sample shuffle sample 0 into a spare slot and write nothing)
         int16_t* cur = scratch + (size_t)(active ? sm : samples + grp) * C::NP;
         gchain_init<G, E, UCD>(ch, cur, n, seed, (uint64_t)(active ? sm : 0), l, T, nullptr, nullptr, kTagT0);
-        const int32_t z = gchain_eval<G, E, UCD>(ch, l, gbase, n, d, ch.tot()[l]);
+        const int32_t z = gchain_eval<G, E, UCD>(ch, l, gbase, n, d, ch.tot()[l], quad);
         if (active && l == 0) Z[sm] = z;
         __syncwarp();
     }
@@ -851,7 +892,7 @@ cudaError_t t0_group_impl(const Instance& I, uint64_t seed, int64_t samples, dou
     uint8_t* base = static_cast<uint8_t*>(ws);
     int64_t* Z = reinterpret_cast<int64_t*>(base + w.z_off);
     int16_t* scratch = reinterpret_cast<int16_t*>(base + w.t0s_off);
-    t0_group_kernel<G, E, UCD><<<(unsigned)blocks, kGThreads, smem, s>>>(tables(I, UCD), I.n, I.d_eff, seed,
+    t0_group_kernel<G, E, UCD><<<(unsigned)blocks, kGThreads, smem, s>>>(tables(I, UCD), I.n, I.d_eff, I.ab85_ok, seed,
                                                                        samples, scratch, Z);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return e;
@@ -922,6 +963,7 @@ cudaError_t sag_impl(Instance& I, const SaLaunch& p, void* ws, cudaStream_t s) {
     cudaError_t e = cudaMemsetAsync(I.best_key, 0xff, sizeof(unsigned long long), s);
     if (e != cudaSuccess) return e;
     SaGArgs a{};
+    a.quad = I.ab85_ok && !getenv("CDD_SA_NO_QUAD");
     a.T = tables(I, UCD);
     a.n = I.n;
     a.d = I.d_eff;
@@ -1046,23 +1088,19 @@ __global__ void sync_level_prepare(double* T, double mu, unsigned long long* key
         }
         ids[k] = (int16_t)j;
         const bool v = k < n;
-        ch.ab()[C::ab_h(k)] = v ? tb.ab16[j] : (uint16_t)0;
+        const uint32_t ab = v ? tb.ab16[j] : 0u;
         ch.pb()[C::pb_b(k)] = v ? tb.p[j] : (uint8_t)0;
         if constexpr (UCD) {
+            ch.ab()[C::ab_h(k)] = (uint16_t)ab;
             ch.xb()[C::pb_b(k)] = v ? tb.x[j] : (uint8_t)0;
             ch.gh()[C::gh_h(k)] = v ? tb.g[j] : (uint16_t)0;
+        } else {
+            ch.a8()[C::rb(k)] = (uint8_t)ab;
+            ch.b8()[C::rb(k)] = (uint8_t)(ab >> 8);
         }
     }
     __syncthreads();
-    if (threadIdx.x < G) {
-        const int l = threadIdx.x;
-        uint32_t tAB = 0, tP = 0;
-        for (int i = 0; i < E; ++i) {
-            tAB += ab_wide(ch.ab()[l * (C::AS / 2) + i]);
-            tP += ch.pb()[l * C::PS + i];
-        }
-        ch.tot()[l] = make_uint2(tAB, tP);
-    }
+    if (threadIdx.x < G) ch.tot()[threadIdx.x] = gchain_lane_totals(ch, (int)threadIdx.x);
     __syncthreads();
     for (int i = threadIdx.x; i < C::BYTES / 16; i += blockDim.x)
         reinterpret_cast<int4*>(image)[i] = reinterpret_cast<const int4*>(buf)[i];
@@ -1127,6 +1165,7 @@ cudaError_t sag_sync_level(Instance& I, const SaLaunch& p, int64_t j, int64_t* l
         if (e != cudaSuccess) return e;
     }
     SaGArgs a{};
+    a.quad = I.ab85_ok && !getenv("CDD_SA_NO_QUAD");
     a.T = tables(I, UCD);
     a.n = I.n;
     a.d = I.d_eff;

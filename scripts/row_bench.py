@@ -8,8 +8,13 @@ bounds it (DESIGN.md §7 / §8): prints one JSON line per row.
   F1  cdd_schedule_batch, n=1000: HBM (2n read + 8n written + 16 bytes per sequence)
   F2  synchronous SA, n=1000: issue (6n per evaluation)
 
-Peaks: MEASURED_PEAKS.json (HBM GB/s, SM max clock); integer issue peak = 128 lane-ops/clk/SM x SMs
-x max clock.  Inputs larger than L2 for the HBM rows (two alternating pools).
+  S4  SA with the insertion / window moves (R11b / R11c), n=1000
+  G   the generic ("wide") path: batched evaluation at n=1000 (warp per sequence) and n=4096 (CTA
+      per sequence), asynchronous SA at n=1000
+
+Peaks: MEASURED_PEAKS.json (HBM GB/s, SM max clock); integer peak = the best measured lane-op rate
+of scripts/int_peak.cu (profiles/r2_int_peak.jsonl) x SMs x max clock.  Inputs larger than L2 for
+the HBM rows (two alternating pools).
 python scripts/row_bench.py"""
 import json
 import os
@@ -44,7 +49,9 @@ def main():
     hbm = float(peaks.get("hbm_gbs", 6454.0))
     sm_mhz = float(peaks.get("sm_max_mhz", 1965.0))
     nsm = torch.cuda.get_device_properties(0).multi_processor_count
-    alu = 128 * nsm * sm_mhz * 1e6 / 1e12  # T int-op/s
+    ip = [json.loads(x) for x in open(os.path.join(ROOT, "profiles", "r2_int_peak.jsonl")) if x.startswith("{")]
+    lane_ops = max(r["lane_ops_per_clk_per_sm"] for r in ip)
+    alu = lane_ops * nsm * sm_mhz * 1e6 / 1e12  # T int-op/s (measured)
 
     def out(row, what, value, unit, achieved, peak, punit, note=""):
         print(json.dumps({"row": row, "what": what, "value": value, "unit": unit,
@@ -97,14 +104,48 @@ def main():
         6 * n * ev / dt / 1e12, alu, "Tint-op/s")
 
     # A13-A14 DPSO
-    n2 = 500
-    i5 = cdd.Instance.from_gen(gen.cdd_instance(n2, 1, 0.6))
-    P, it = 8192, 200
-    sw = cdd.Dpso(i5, P, it, seed=4)
-    dt = timed(lambda r=0: sw.run(), reps=3)
-    ev = P * (it + 1)
-    out("A13-A14", f"DPSO n={n2}, {P} particles x {it} iterations", ev / dt, "particle-evals/s",
-        6 * n2 * ev / dt / 1e12, alu, "Tint-op/s", "per iteration: F1-F3 + evaluation + swarm best")
+    for n2 in (100, 500, 1000):
+        i5 = cdd.Instance.from_gen(gen.cdd_instance(n2, 1, 0.6))
+        P, it = 8192, 200
+        sw = cdd.Dpso(i5, P, it, seed=4)
+        dt = timed(lambda r=0: sw.run(), reps=3)
+        ev = P * (it + 1)
+        out("A13-A14", f"DPSO n={n2}, {P} particles x {it} iterations", ev / dt, "particle-evals/s",
+            6 * n2 * ev / dt / 1e12, alu, "Tint-op/s", "per iteration: F1-F3 + evaluation + swarm best")
+
+    # S4: the other moves on the headline instance
+    for mv in ("insert", "window", "swap"):
+        C, S = 65536, 1000
+        t0 = cdd.sa_t0(ic, seed=1, samples=T0)
+        ws = cdd.sa_run(ic, C, S, seed=1, T0_dev=t0, move=mv)["workspace"]
+        dt = timed(lambda r=0: cdd.sa_run(ic, C, S, seed=1, T0_dev=t0, workspace=ws, move=mv), reps=3)
+        ev = C * (S + 1)
+        out("S4", f"SA cdd n={n} move={mv}, {C} chains x {S} steps", ev / dt, "evals/s",
+            6 * n * ev / dt / 1e12, alu, "Tint-op/s")
+
+    # G: generic path (values outside the packed ranges)
+    import numpy as np
+
+    rng = np.random.default_rng(5)
+    for nw, batch in ((1000, 1 << 18), (4096, 1 << 14)):
+        P = rng.integers(1, 1001, nw).astype(np.int32)
+        a = rng.integers(1, 10001, nw).astype(np.int32)
+        b = rng.integers(1, 10001, nw).astype(np.int32)
+        iw = cdd.Instance(P, a, b, int(0.4 * int(P.sum())))
+        assert iw.wide
+        pw = [gen.random_perms_device(batch, nw, seed=s, ld=nw) for s in (3, 4)]
+        ow = torch.empty(batch, dtype=torch.int64, device="cuda")
+        dt = timed(lambda r=0: cdd.cdd_eval_batch(iw, pw[r & 1], ow), reps=5)
+        out("G", f"generic cdd_eval_batch n={nw} (p<=1000, alpha,beta<=1e4), {batch} sequences", batch / dt,
+            "evals/s", batch * (2 * nw + 8) / dt / 1e9, hbm, "GB/s",
+            "int64 arithmetic, int4 record gathers from L1/L2 (3 passes)")
+        if nw == 1000:
+            C, S = 16384, 200
+            ws = cdd.sa_run(iw, C, S, seed=1, T0=1e9)["workspace"]
+            dt = timed(lambda r=0: cdd.sa_run(iw, C, S, seed=1, T0=1e9, workspace=ws), reps=3)
+            ev = C * (S + 1)
+            out("G", f"generic SA n={nw}, {C} chains x {S} steps", ev / dt, "evals/s",
+                6 * nw * ev / dt / 1e12, alu, "Tint-op/s", "one warp per chain, ids in L2")
 
 
 if __name__ == "__main__":

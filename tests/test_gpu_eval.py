@@ -221,10 +221,13 @@ def test_instance_argument_errors(lib):
     with pytest.raises(lib.CddError):
         lib.Instance([0, 1], [1, 1], [1, 1], 3)          # p_i >= 1
     with pytest.raises(lib.CddError):
-        lib.Instance([1] * 1025, [1] * 1025, [1] * 1025, 3)  # n <= 1024
-    with pytest.raises(lib.CddError) as e:
-        lib.Instance([1000] * 10, [1000] * 10, [1] * 10, 3)
+        lib.Instance([1] * 32768, [1] * 32768, [1] * 32768, 3)  # n <= 32767 (int16 job ids)
+    with pytest.raises(lib.CddError) as e:  # a penalty could reach 2^62 (R20)
+        lib.Instance([2**31 - 1] * 10, [2**31 - 1] * 10, [1] * 10, 3)
     assert e.value.code == lib.CDD_ERANGE
+    # outside the packed records, inside int64: the generic path (round 1 refused these)
+    assert lib.Instance([1000] * 10, [1000] * 10, [1] * 10, 3).query()["generic"]
+    assert lib.Instance([1] * 1025, [1] * 1025, [1] * 1025, 3).query()["generic"]
     inst = gen.cdd_instance(20, 1, 0.4)
     ins = lib.Instance(inst.P, inst.alpha, inst.beta, inst.d)
     with pytest.raises(lib.CddError):

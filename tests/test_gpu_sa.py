@@ -256,10 +256,11 @@ def test_edge_instances_trace_parity(lib, n, kw, problem, lanes):
         pytest.skip("lanes=4 needs n <= 256")
     inst = gen.ranged_instance(n, 9, problem=problem, **kw)
     chains = 24
-    if problem == "ucddcp" and not lib.Instance.from_gen(inst).query()["has_ucddcp"]:
-        # M, P-M, gamma do not fit the packed UCDDCP record: refused, the CDD side still works
+    if problem == "ucddcp" and lib.Instance.from_gen(inst).query()["ucddcp_generic"] and lanes in (4, 8, 16):
+        # M, P-M, gamma do not fit the packed UCDDCP record: the UCDDCP runs on the generic path
+        # (one warp per chain), the group layouts refuse it
         with pytest.raises(lib.CddError):
-            lib.sa_run(lib.Instance.from_gen(inst), 4, 10, problem="ucddcp", T0=1.0)
+            lib.sa_run(lib.Instance.from_gen(inst), 4, 10, problem="ucddcp", T0=1.0, lanes=lanes)
         return
     ins, res, (pen, perm, gid), pr, p, T0 = _run_both(lib, inst, problem, chains, 120, 31 + n,
                                                      samples=200, lanes=lanes)
