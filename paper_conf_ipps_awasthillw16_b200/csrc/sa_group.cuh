@@ -397,7 +397,7 @@ __device__ __forceinline__ int32_t gchain_eval_cdd(const GChain<G, E>& ch, int l
     const bool amode = l < Ls;
     const uint8_t* xrow = (amode ? ch.a8() : ch.b8()) + l * C::RS;
     const uint8_t* prow = ch.pb() + l * C::RS;
-    constexpr int CH = E >= 16 ? 16 : E;  // positions per chunk
+    constexpr int CH = E >= 16 ? 16 : E;  // positions per chunk (32 measured: same speed)
     uint32_t s = 0, acc = 0;
     if (quad) {
         // per quad: byte-wise exclusive prefixes [0, x0, x0+x1, x0+x1+x2] by one IMAD, their dot
