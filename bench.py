@@ -248,6 +248,11 @@ def main():
     torch.cuda.set_device(local)
     if world > 1:
         backend = os.environ.get("CDD_BENCH_BACKEND", "nccl")
+        # the communicator log (ranks, devices, transports: NVLink / NVLS) on stderr, so the JSON
+        # line stays alone on stdout
+        os.environ.setdefault("NCCL_DEBUG", "INFO")
+        os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+        os.environ.setdefault("NCCL_DEBUG_FILE", "/dev/stderr")
         if backend == "nccl":
             dist.init_process_group("nccl", device_id=torch.device("cuda", local))
         else:

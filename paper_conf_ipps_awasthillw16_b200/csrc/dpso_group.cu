@@ -502,6 +502,14 @@ __global__ void __launch_bounds__(DgSmem<DG, E, UCD>::THREADS, 1) dpsog_iter_ker
     // from the first iteration of the launch to the last (loaded / stored once per launch)
     const bool resident = groups >= a.particles;
     const int64_t i0r = (int64_t)blockIdx.x * per_cta + wib * PPW;
+    // every slot starts from the identity (valid ids < NP): the slots past the swarm are evaluated
+    // too (their results are discarded) and must not gather outside the tables
+    for (int p = 0; p < PPW; ++p)
+        for (int k = lane; k < NP; k += 32) {
+            ids_of(p)[k] = (uint16_t)k;
+            inv_of(p)[k] = (uint16_t)k;
+        }
+    __syncwarp();
     if (resident)
         for (int p = 0; p < PPW; ++p)
             if (i0r + p < a.particles) {

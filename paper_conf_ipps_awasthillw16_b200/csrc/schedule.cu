@@ -56,8 +56,10 @@ __device__ __forceinline__ int64_t warp_sum64(int64_t v) {
 // Shared-memory layout (dynamic): the instance tables by job id (ab u32, p u8 [, M u8, X u8,
 // gamma u16], each array padded to 16 bytes), then per warp: the sequence's ids in lane segments
 // of E positions (E = pow2 >= ceil(n/32), segments padded by 16 bytes), and the output staging
-// C (int64) [and X (int32)] in lane segments padded by one element, so that the lane-contiguous
-// compute writes and the coalesced copy-out reads are both (nearly) conflict free.
+// C [and X] (int32) in lane segments padded by one element, so that the lane-contiguous compute
+// writes and the coalesced copy-out reads are both (nearly) conflict free.  C is staged relative
+// to a per-sequence int64 base (CDD: the start time; UCDDCP: d), |C - base| <= sum P < 2^31: half
+// the shared memory of int64 staging, so more warps fit per SM.
 struct SchedLayout {
     int n, E, lE;
     uint32_t tab_bytes, ids_off, c_off, x_off, warp_bytes, total;
@@ -73,15 +75,18 @@ __host__ __device__ inline SchedLayout sched_layout(int n, bool ucd, int warps) 
     L.tab_bytes = al16(4 * (N + 1)) + al16(N + 1) + (ucd ? al16(N + 1) + al16(N + 1) + al16(2 * (N + 1)) : 0u);
     L.ids_off = 0;
     L.c_off = al16(32u * (2u * L.E + 16u));
-    L.x_off = L.c_off + al16(32u * 8u * (L.E + 1u));
+    L.x_off = L.c_off + al16(32u * 4u * (L.E + 1u));
     L.warp_bytes = L.x_off + (ucd ? al16(32u * 4u * (L.E + 1u)) : 0u);
     L.total = L.tab_bytes + (uint32_t)warps * L.warp_bytes;
     return L;
 }
 constexpr int kSchedWarps = 4;
+#ifndef CDD_SCHED_MINB
+#define CDD_SCHED_MINB 4
+#endif
 
 template <bool UCD, int E>
-__global__ void __launch_bounds__(kSchedWarps * 32, 4) schedule_kernel(SchedArgs a) {
+__global__ void __launch_bounds__(kSchedWarps * 32, CDD_SCHED_MINB) schedule_kernel(SchedArgs a) {
     extern __shared__ __align__(16) uint8_t smem[];
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
     const int n = a.n;
@@ -109,7 +114,7 @@ __global__ void __launch_bounds__(kSchedWarps * 32, 4) schedule_kernel(SchedArgs
     }
     uint8_t* wbase = smem + Ly.tab_bytes + (size_t)wib * Ly.warp_bytes;
     uint16_t* ids_s = reinterpret_cast<uint16_t*>(wbase + Ly.ids_off);
-    int64_t* C_s = reinterpret_cast<int64_t*>(wbase + Ly.c_off);
+    int32_t* C_s = reinterpret_cast<int32_t*>(wbase + Ly.c_off);
     int32_t* X_s = reinterpret_cast<int32_t*>(wbase + Ly.x_off);
     const int IS = E + 8, CS = E + 1;  // segment strides (elements)
     const int k_lo = lane * E;
@@ -117,7 +122,7 @@ __global__ void __launch_bounds__(kSchedWarps * 32, 4) schedule_kernel(SchedArgs
     for (int k = n + lane; k < 32 * E; k += 32) ids_s[(k >> lE) * IS + (k & (E - 1))] = (uint16_t)n;
     __syncthreads();
     const uint16_t* myids = ids_s + lane * IS;
-    int64_t* myC = C_s + lane * CS;
+    int32_t* myC = C_s + lane * CS;
     int32_t* myX = X_s + lane * CS;
     const int64_t warps = (int64_t)gridDim.x * kSchedWarps;
     bool bad = false;
@@ -240,14 +245,15 @@ __global__ void __launch_bounds__(kSchedWarps * 32, 4) schedule_kernel(SchedArgs
         if constexpr (!UCD) {
             const int64_t D = min((int64_t)Ck0, a.d);
             st = a.d - D;  // start of the first job
-            int64_t c = st + Pb;
+            // C_k = st + c_k with c_k the prefix from time 0; D - c_k compares against the due date
+            int32_t c = Pb;
+            const int32_t Dl = (int32_t)D;  // D <= C_{k0} <= sum P
             #pragma unroll
         for (int i = 0; i < E; ++i) {
                 const uint32_t r = rec_r(i);
                 c += rec_p(i);
                 myC[i] = c;
-                pen += (int64_t)(r & 0xffffu) * max((int64_t)0, a.d - c) +
-                       (int64_t)(r >> 16) * max((int64_t)0, c - a.d);
+                pen += (int64_t)(r & 0xffffu) * max(0, Dl - c) + (int64_t)(r >> 16) * max(0, c - Dl);
             }
         } else {
             // compression decisions and the lane totals of p'
@@ -287,10 +293,10 @@ __global__ void __launch_bounds__(kSchedWarps * 32, 4) schedule_kernel(SchedArgs
                 const uint32_t r = t_ab[j];
                 const int32_t xk = myX[i];
                 q += (int32_t)t_m[j] + (int32_t)t_x[j] - xk;
-                const int64_t c = a.d - (int64_t)(Qk0 - q);
+                const int32_t c = q - Qk0;  // C_k - d
                 myC[i] = c;
-                pen += (int64_t)(r & 0xffffu) * max((int64_t)0, a.d - c) +
-                       (int64_t)(r >> 16) * max((int64_t)0, c - a.d) + (int64_t)t_g[j] * xk;
+                pen += (int64_t)(r & 0xffffu) * max(0, -c) + (int64_t)(r >> 16) * max(0, c) +
+                       (int64_t)t_g[j] * xk;
             }
         }
         pen = warp_sum64(pen);
@@ -299,15 +305,16 @@ __global__ void __launch_bounds__(kSchedWarps * 32, 4) schedule_kernel(SchedArgs
             a.pen[row] = pen;
         }
         __syncwarp();
-        // coalesced copy-out of the staged rows
+        // coalesced copy-out of the staged rows (the int64 base added here)
         int64_t* Crow = a.C + row * (int64_t)n;
+        const int64_t cb = UCD ? a.d : st;
         if (pairs) {  // 16-byte streaming stores of position pairs (same lane segment: E even)
             for (int k = 2 * lane; k < n; k += 64) {
                 const int idx = (k >> lE) * CS + (k & (E - 1));
-                __stcs(reinterpret_cast<longlong2*>(Crow + k), make_longlong2(C_s[idx], C_s[idx + 1]));
+                __stcs(reinterpret_cast<longlong2*>(Crow + k), make_longlong2(cb + C_s[idx], cb + C_s[idx + 1]));
             }
         } else {
-            for (int k = lane; k < n; k += 32) Crow[k] = C_s[(k >> lE) * CS + (k & (E - 1))];
+            for (int k = lane; k < n; k += 32) Crow[k] = cb + C_s[(k >> lE) * CS + (k & (E - 1))];
         }
         if constexpr (UCD) {
             int32_t* Xrow = a.X + row * (int64_t)n;
