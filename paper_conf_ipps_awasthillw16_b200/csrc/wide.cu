@@ -151,22 +151,69 @@ __device__ __forceinline__ WideSplit wide_split(const WideTab& T, int n, int t, 
 
 // Optimal penalty of the group's sequence: eq. (1) at D = min(C_{k0}, d) (CDD) or eq. (2) with the
 // Property 1/2 weights (UCDDCP, d >= sum P).  Every thread of the group returns it.
+// CDD in one gather pass: besides the sums, each thread keeps DA = sum alpha_k c_k and
+// DB = sum beta_k c_k over its segment (c_k = completion time from the segment start), so a segment
+// wholly before the due date D contributes A (D - C_start) - DA, one wholly after it
+// B (C_start - D) + DB; only the thread whose segment holds D walks it again (and the owner of
+// k0, for C_{k0}) -- the split F(C) = F(C_m') + integral of the fast kernels.
+template <int TH, class IdAt>
+__device__ __forceinline__ long long wide_eval_cdd(const WideTab& T, int n, long long d, int t, IdAt&& id_at,
+                                                   long long* sm) {
+    const int S = (n + TH - 1) / TH;
+    const int ka = min(n, t * S), kb = min(n, ka + S);
+    long long Pt = 0, At = 0, Bt = 0, DA = 0, DB = 0;
+    for (int k = ka; k < kb; ++k) {
+        const int4 r = __ldg(T.w0 + id_at(k));
+        Pt += r.x;
+        At += r.y;
+        Bt += r.z;
+        DA += (long long)r.y * Pt;
+        DB += (long long)r.z * Pt;
+    }
+    long long Ptot, Atot, Btot;
+    const long long Pex = wgroup_excl_scan<TH>(Pt, Ptot, sm);
+    const long long Aex = wgroup_excl_scan<TH>(At, Atot, sm);
+    const long long Bex = wgroup_excl_scan<TH>(Bt, Btot, sm);
+    // k0 = max{k : S_k <= Btot} (a prefix): the owner walks its segment for C_{k0}
+    const int own = wgroup_max<TH>((ka < kb && Aex + Bex <= Btot) ? t : 0, sm);
+    long long cc = 0;
+    if (t == own) {
+        long long s = Aex + Bex, c = Pex;
+        for (int k = ka; k < kb; ++k) {
+            const int4 r = __ldg(T.w0 + id_at(k));
+            c += r.x;
+            if (s <= Btot) cc = c;
+            s += (long long)r.y + r.z;
+        }
+    }
+    const long long D = min(wgroup_bcast<TH>(cc, own, sm), d);
+    long long z = 0;
+    if (ka < kb) {
+        if (Pex + Pt <= D) {
+            z = At * (D - Pex) - DA;
+        } else if (Pex >= D) {
+            z = Bt * (Pex - D) + DB;
+        } else {  // the segment that holds D
+            long long c = Pex;
+            for (int k = ka; k < kb; ++k) {
+                const int4 r = __ldg(T.w0 + id_at(k));
+                c += r.x;
+                z += D > c ? (long long)r.y * (D - c) : (long long)r.z * (c - D);
+            }
+        }
+    }
+    return wgroup_sum<TH>(z, sm);
+}
+
 template <int TH, bool UCD, class IdAt>
 __device__ __forceinline__ long long wide_eval(const WideTab& T, int n, long long d, int t, IdAt&& id_at,
                                                long long* sm) {
+    if constexpr (!UCD) return wide_eval_cdd<TH>(T, n, d, t, id_at, sm);
     const WideSplit w = wide_split<TH>(T, n, t, id_at, sm);
     const int S = (n + TH - 1) / TH;
     const int ka = min(n, t * S), kb = min(n, ka + S);
     long long z = 0;
-    if constexpr (!UCD) {
-        const long long D = min(w.Ck0, d);
-        long long c = w.Pex;
-        for (int k = ka; k < kb; ++k) {
-            const int4 r = __ldg(T.w0 + id_at(k));
-            c += r.x;
-            z += D > c ? (long long)r.y * (D - c) : (long long)r.z * (c - D);
-        }
-    } else {
+    {
         long long a = w.Aex, b = w.Btot - w.Bex;
         for (int k = ka; k < kb; ++k) {
             const int j = id_at(k);

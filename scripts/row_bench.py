@@ -15,7 +15,7 @@ bounds it (DESIGN.md §7 / §8): prints one JSON line per row.
 Peaks: MEASURED_PEAKS.json (HBM GB/s, SM max clock); integer peak = the best measured lane-op rate
 of scripts/int_peak.cu (profiles/r2_int_peak.jsonl) x SMs x max clock.  Inputs larger than L2 for
 the HBM rows (two alternating pools).
-python scripts/row_bench.py"""
+python scripts/row_bench.py [ROW ...]   (default: every row; e.g. `G S4`)"""
 import json
 import os
 import sys
@@ -44,6 +44,11 @@ def timed(fn, reps=5):
 
 
 def main():
+    sel = set(sys.argv[1:])
+
+    def want(row):
+        return not sel or row in sel
+
     peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json"))) if os.path.exists(
         os.path.join(ROOT, "MEASURED_PEAKS.json")) else {}
     hbm = float(peaks.get("hbm_gbs", 6454.0))
@@ -64,7 +69,8 @@ def main():
     o = torch.empty(rows, dtype=torch.int64, device="cuda")
     ic = cdd.Instance.from_gen(gen.cdd_instance(n, 1, 0.4))
     iu = cdd.Instance.from_gen(gen.ucddcp_instance(n, 1))
-    for name, ins, fn in (("cdd_eval_batch", ic, cdd.cdd_eval_batch), ("ucddcp_eval_batch", iu, cdd.ucddcp_eval_batch)):
+    for name, ins, fn in ((("cdd_eval_batch", ic, cdd.cdd_eval_batch), ("ucddcp_eval_batch", iu, cdd.ucddcp_eval_batch))
+                          if want("A7") else ()):
         dt = timed(lambda r=0: fn(ins, pools[r & 1], o), reps=9)
         gbs = rows * (2 * n + 8) / dt / 1e9
         out("A7" if name.startswith("cdd") else "A6/A7", f"{name} n={n}, 2^20 sequences", rows / dt,
@@ -75,18 +81,20 @@ def main():
     # F1 schedules: C int64 [B, n] written, sequences read
     B = 1 << 17
     sp = pools[0][:B]
-    dt = timed(lambda r=0: cdd.cdd_schedule_batch(ic, sp), reps=5)
-    out("F1", f"cdd_schedule_batch n={n}, 2^17 sequences", B / dt, "schedules/s",
-        B * (2 * n + 8 * n + 16) / dt / 1e9, hbm, "GB/s", "C int64 [B, n] written + start + penalty")
+    if want("F1"):
+        dt = timed(lambda r=0: cdd.cdd_schedule_batch(ic, sp), reps=5)
+        out("F1", f"cdd_schedule_batch n={n}, 2^17 sequences", B / dt, "schedules/s",
+            B * (2 * n + 8 * n + 16) / dt / 1e9, hbm, "GB/s", "C int64 [B, n] written + start + penalty")
 
     # A8 T0
     T0 = 5000
-    dt = timed(lambda r=0: cdd.sa_t0(ic, seed=r, samples=T0), reps=9)
-    out("A8", f"T0 rule, {T0} samples, n={n}", T0 / dt, "samples/s", 6 * n * T0 / dt / 1e12, alu,
-        "Tint-op/s", "one launch pair: small grid (5000 warps), latency-bound")
+    if want("A8"):
+        dt = timed(lambda r=0: cdd.sa_t0(ic, seed=r, samples=T0), reps=9)
+        out("A8", f"T0 rule, {T0} samples, n={n}", T0 / dt, "samples/s", 6 * n * T0 / dt / 1e12, alu,
+            "Tint-op/s", "one launch pair: small grid (5000 warps), latency-bound")
 
     # A9-A11 SA (CDD and UCDDCP)
-    for prob, ins, ops in (("cdd", ic, 6), ("ucddcp", iu, 9)):
+    for prob, ins, ops in (("cdd", ic, 6), ("ucddcp", iu, 9)) if want("A9") else ():
         C, S = 65536, 1000
         t0 = cdd.sa_t0(ins, problem=prob, seed=1, samples=T0)
         ws = cdd.sa_run(ins, C, S, problem=prob, seed=1, T0_dev=t0)["workspace"]
@@ -97,14 +105,15 @@ def main():
 
     # F2 synchronous SA
     C, M, L = 65536, 50, 20
-    ss = cdd.SaSync(ic, C, M, L, seed=3, t0_samples=T0, level_min=False)
-    dt = timed(lambda r=0: ss.run(), reps=3)
-    ev = C * M * L
-    out("F2", f"synchronous SA n={n}, {C} chains, M={M} x {L} levels", ev / dt, "evals/s",
-        6 * n * ev / dt / 1e12, alu, "Tint-op/s")
+    if want("F2"):
+        ss = cdd.SaSync(ic, C, M, L, seed=3, t0_samples=T0, level_min=False)
+        dt = timed(lambda r=0: ss.run(), reps=3)
+        ev = C * M * L
+        out("F2", f"synchronous SA n={n}, {C} chains, M={M} x {L} levels", ev / dt, "evals/s",
+            6 * n * ev / dt / 1e12, alu, "Tint-op/s")
 
     # A13-A14 DPSO
-    for n2 in (100, 500, 1000):
+    for n2 in (100, 500, 1000) if want("A13") else ():
         i5 = cdd.Instance.from_gen(gen.cdd_instance(n2, 1, 0.6))
         P, it = 8192, 200
         sw = cdd.Dpso(i5, P, it, seed=4)
@@ -114,7 +123,7 @@ def main():
             6 * n2 * ev / dt / 1e12, alu, "Tint-op/s", "per iteration: F1-F3 + evaluation + swarm best")
 
     # S4: the other moves on the headline instance
-    for mv in ("insert", "window", "swap"):
+    for mv in ("insert", "window", "swap") if want("S4") else ():
         C, S = 65536, 1000
         t0 = cdd.sa_t0(ic, seed=1, samples=T0)
         ws = cdd.sa_run(ic, C, S, seed=1, T0_dev=t0, move=mv)["workspace"]
@@ -127,7 +136,7 @@ def main():
     import numpy as np
 
     rng = np.random.default_rng(5)
-    for nw, batch in ((1000, 1 << 18), (4096, 1 << 14)):
+    for nw, batch in ((1000, 1 << 18), (4096, 1 << 14)) if want("G") else ():
         P = rng.integers(1, 1001, nw).astype(np.int32)
         a = rng.integers(1, 10001, nw).astype(np.int32)
         b = rng.integers(1, 10001, nw).astype(np.int32)
