@@ -447,7 +447,7 @@ constexpr size_t kAlign = 256;
 inline size_t align_up(size_t x) { return (x + kAlign - 1) / kAlign * kAlign; }
 
 struct DpWs {
-    size_t pos, inv, pb, zb, gkey, gperm, counter, ctakeys, total;
+    size_t pos, inv, pb, zb, gkey, gperm, counter, slots, total;
 };
 
 DpWs dp_layout(int np, int64_t N) {
@@ -459,8 +459,10 @@ DpWs dp_layout(int np, int64_t N) {
     w.gkey = align_up(w.zb + (size_t)N * 4);
     w.gperm = align_up(w.gkey + 16);
     w.counter = align_up(w.gperm + (size_t)2 * np * 2);
-    w.ctakeys = align_up(w.counter + 16);
-    w.total = align_up(w.ctakeys + sizeof(unsigned long long) * kDpsoMaxCtas);
+    w.slots = align_up(w.counter + 32);  // counters [4], the group publish's running keys [2]
+    // one row per CTA and parity for the group layout's publish (a CTA holds >= 4 particles)
+    const int64_t ctas = std::min<int64_t>(kDpsoMaxCtas, (N + 3) / 4 + 1);
+    w.total = align_up(w.slots + (size_t)2 * ctas * np * 2);
     return w;
 }
 
@@ -481,7 +483,7 @@ DpsoWsPtrs ws_ptrs(const Instance& I, const DpsoLaunch& p, void* ws) {
     r.gkey = reinterpret_cast<unsigned long long*>(b + w.gkey);
     r.gperm = reinterpret_cast<int16_t*>(b + w.gperm);
     r.counter = reinterpret_cast<unsigned int*>(b + w.counter);
-    r.ctakeys = reinterpret_cast<unsigned long long*>(b + w.ctakeys);
+    r.slots = reinterpret_cast<int16_t*>(b + w.slots);
     r.np = np;
     return r;
 }

@@ -47,8 +47,11 @@ struct DgArgs {
     int64_t pper;
     uint8_t* const* pregions;
     int* err;
-    unsigned int* counter;      // [0] CTA arrivals, [3] iterations whose swarm best is released
-    unsigned long long* ctakeys;  // [gridDim]: each CTA's minimum key of the current publish
+    unsigned int* counter;      // [0] CTA arrivals, [3] iterations whose swarm best is released;
+                                // [1], [2]: arrivals per parity, [4..7]: running keys per parity
+                                // (single-GPU publish)
+    int16_t* slots;             // [2][gridDim][np]: each CTA's best personal-best row per parity
+    unsigned long long* fkey;   // [2] = counter + 4: the single-GPU publish's running minima
     int64_t* trace;
     int np;
     bool quad;  // CDD with max(alpha, beta) <= 85 (the evaluator's quad pass)
@@ -98,47 +101,45 @@ __device__ __forceinline__ unsigned long long warp_min64(unsigned long long v) {
 }
 
 // Alg. 2 line 5 for the swarm after iteration `done` (0: after line 2): CTA min of the particles'
-// keys, one atomicMin per CTA on gkey[nxt], and the last CTA to arrive copies the winner's personal
-// best to gperm[nxt] (exchanging it across GPUs first when pw > 1), re-arms gkey[cur] and releases
-// counter[3] = done.
+// keys, one atomicMin per CTA on gkey[nxt] (no round trip: a reduction in L2), the arrival, and the
+// last CTA to arrive copies the winner's personal best to gperm[nxt] (exchanging it across GPUs
+// first when pw > 1), re-arms gkey[cur] and releases counter[3] = done.  The swarm best of Alg. 2 is
+// the minimum over the personal bests, which never increase, so an unchanged key means an unchanged
+// row: then the copy is skipped (every CTA still holds that row in shared memory), except on the
+// last publish of a launch (`final`), whose row the next launch and the end kernel read.
 template <int W>
 __device__ void dg_publish(const DgArgs& a, unsigned long long wkey, int nxt, int cur, bool rearm, uint32_t done,
-                           bool trace) {
-    __shared__ unsigned long long s_key[W];
+                           bool trace, bool final) {
+    __shared__ unsigned long long s_key[2];
+    __shared__ unsigned long long s_wkey[W];
     __shared__ bool s_last;
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
     const int nw = (int)(blockDim.x >> 5);
     wkey = warp_min64(wkey);
-    if (lane == 0) s_key[wib] = wkey;
+    if (lane == 0) s_wkey[wib] = wkey;
     __syncthreads();  // the CTA's personal-best writes happen before thread 0's (cumulative) fence
     if (threadIdx.x == 0) {
-        unsigned long long mk = s_key[0];
-        for (int i = 1; i < nw; ++i) mk = s_key[i] < mk ? s_key[i] : mk;
-        // one L2 round trip per CTA: its minimum to its own slot, then the arrival
-        a.ctakeys[blockIdx.x] = mk;
+        unsigned long long mk = s_wkey[0];
+        for (int i = 1; i < nw; ++i) mk = s_wkey[i] < mk ? s_wkey[i] : mk;
+        if (mk != ULLONG_MAX) atomicMin(a.gkey + nxt, mk);
         __threadfence();
         const unsigned int prev = atomicAdd(a.counter, 1u);
         s_last = prev == gridDim.x - 1;
-        if (s_last) __threadfence();  // every other CTA's writes (fenced before its arrival) visible
+        if (s_last) {
+            __threadfence();  // every other CTA's writes (fenced before its arrival) visible
+            s_key[0] = __ldcg(a.gkey + nxt);
+            s_key[1] = rearm ? __ldcg(a.gkey + cur) : ULLONG_MAX;  // the previous release's key
+        }
     }
     __syncthreads();
     if (s_last) {
-        // the swarm minimum over the CTAs' slots
-        unsigned long long m = ULLONG_MAX;
-        for (int i = threadIdx.x; i < (int)gridDim.x; i += blockDim.x) {
-            const unsigned long long v = __ldcg(a.ctakeys + i);
-            m = v < m ? v : m;
-        }
-        m = warp_min64(m);
-        __syncthreads();
-        if (lane == 0) s_key[wib] = m;
-        __syncthreads();
-        unsigned long long k = s_key[0];
-        for (int i = 1; i < nw; ++i) k = s_key[i] < k ? s_key[i] : k;
+        const unsigned long long k = s_key[0];
+        const bool copy = final || a.pw > 1 || k != s_key[1];
         const int64_t li = (int64_t)((k & 0xffffffffull) - a.offset);
         const int16_t* src = a.pb + (size_t)li * a.np;
         int16_t* dst = a.gperm + (size_t)nxt * a.np;
-        for (int i = threadIdx.x; i < a.np; i += blockDim.x) dst[i] = __ldcg(src + i);
+        if (copy)
+            for (int i = threadIdx.x; i < a.np; i += blockDim.x) dst[i] = __ldcg(src + i);
         unsigned long long gk = k;
         if (a.pw > 1) {
             __syncthreads();
@@ -170,15 +171,132 @@ __device__ __forceinline__ uint32_t dg_acquire(const unsigned int* p) {
 }
 
 template <int NP>
-__device__ __forceinline__ void dg_cta_stage(const DgArgs& a, uint16_t* g_sm, uint32_t t) {
+__device__ __forceinline__ void dg_cta_stage(const DgArgs& a, uint16_t* g_sm, uint32_t t, unsigned long long* s_gk) {
     __syncthreads();
     if (threadIdx.x < 32) {
-        if (threadIdx.x == 0)
-            while ((int32_t)(dg_acquire(a.counter + 3) - t) < 0) __nanosleep(32);
-        __syncwarp();
-        const int16_t* src = a.gperm + (size_t)(t & 1) * a.np;
-        for (int o = 8 * (int)threadIdx.x; o < NP; o += 256)
-            *reinterpret_cast<uint4*>(g_sm + o) = __ldcg(reinterpret_cast<const uint4*>(src + o));
+        unsigned long long k = 0;
+        if (threadIdx.x == 0) {
+            while ((int32_t)(dg_acquire(a.counter + 3) - t) < 0) {
+            }
+            k = __ldcg(a.gkey + (t & 1));
+        }
+        k = __shfl_sync(kFull, k, 0);
+        // the swarm best row changes only with its key (the copy of an unchanged row is skipped)
+        if (k != *s_gk) {
+            const int16_t* src = a.gperm + (size_t)(t & 1) * a.np;
+            for (int o = 8 * (int)threadIdx.x; o < NP; o += 256)
+                *reinterpret_cast<uint4*>(g_sm + o) = __ldcg(reinterpret_cast<const uint4*>(src + o));
+            __syncwarp();
+            if (threadIdx.x == 0) *s_gk = k;
+        }
+    }
+    __syncthreads();
+}
+
+// Single-GPU publish (no last-CTA step on the critical path).  Every CTA keeps the row of its own
+// best key in slots[parity][cta] (rewritten only when that key changes, before the arrival), adds
+// the key to gkey[nxt] by atomicMin and arrives on the parity's counter; the waiting CTAs see the
+// count, read the swarm key and copy the row from the winner's slot.  Slot rows of a parity are
+// rewritten two publishes later, after every CTA has passed the publish in between, i.e. after
+// every CTA has read them.  The keys go to fkey[parity], which is never re-armed inside a launch:
+// the minimum over the personal bests never increases, so the running minimum of a parity is the
+// swarm best of its latest publish (fkey only ever holds keys of this launch's particles; gkey,
+// which a host-side exchange may overwrite between launches, is read at the launch's first stage
+// only).  The last publish of a launch (`final`) writes gkey[nxt] and gperm[nxt], releases
+// counter[3] (the end kernel, the next launch and the multi-GPU protocol read those) and re-arms
+// the parity counters and fkey for the next launch.
+__device__ __forceinline__ unsigned int dg_target(int64_t done, int64_t t0) {
+    return (unsigned int)((((done - (t0 + 1)) >> 1) + 1) * (int64_t)gridDim.x);
+}
+__device__ __forceinline__ int dg_cta_of(const DgArgs& a, unsigned long long k, int per_cta) {
+    const int64_t li = (int64_t)((k & 0xffffffffull) - a.offset);
+    return (int)((li / per_cta) % (int64_t)gridDim.x);
+}
+
+template <int W>
+__device__ void dg_publish_fast(const DgArgs& a, unsigned long long wkey, int nxt, int64_t done, int64_t t0,
+                                bool final, unsigned long long* s_slot, int per_cta) {
+    __shared__ unsigned long long s_wk[W];
+    __shared__ unsigned long long s_mk;
+    __shared__ bool s_last;
+    const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+    const int nw = (int)(blockDim.x >> 5);
+    wkey = warp_min64(wkey);
+    if (lane == 0) s_wk[wib] = wkey;
+    __syncthreads();  // also: the CTA's personal-best rows are written
+    if (threadIdx.x == 0) {
+        unsigned long long mk = s_wk[0];
+        for (int i = 1; i < nw; ++i) mk = s_wk[i] < mk ? s_wk[i] : mk;
+        s_mk = mk;
+    }
+    __syncthreads();
+    const unsigned long long mk = s_mk;
+    int16_t* slot = a.slots + ((size_t)nxt * gridDim.x + blockIdx.x) * a.np;
+    if (mk != ULLONG_MAX && mk != s_slot[nxt]) {  // CTA-uniform
+        const int64_t li = (int64_t)((mk & 0xffffffffull) - a.offset);
+        const uint4* src = reinterpret_cast<const uint4*>(a.pb + (size_t)li * a.np);
+        for (int o = threadIdx.x; o < a.np / 8; o += blockDim.x) reinterpret_cast<uint4*>(slot)[o] = __ldcg(src + o);
+        __syncthreads();
+        if (threadIdx.x == 0) s_slot[nxt] = mk;
+    }
+    if (threadIdx.x == 0) {
+        if (mk != ULLONG_MAX) atomicMin(a.fkey + nxt, mk);
+        __threadfence();
+        if (!final) {
+            atomicAdd(a.counter + 1 + nxt, 1u);
+        } else {
+            const unsigned int prev = atomicAdd(a.counter + 1 + nxt, 1u);
+            s_last = prev + 1u == dg_target(done, t0);
+        }
+    }
+    if (!final) return;
+    __syncthreads();
+    if (!s_last) return;
+    __shared__ unsigned long long s_k;
+    if (threadIdx.x == 0) {
+        __threadfence();
+        s_k = __ldcg(a.fkey + nxt);
+    }
+    __syncthreads();
+    const unsigned long long k = s_k;
+    const uint4* src = reinterpret_cast<const uint4*>(a.slots + ((size_t)nxt * gridDim.x + dg_cta_of(a, k, per_cta)) * a.np);
+    for (int o = threadIdx.x; o < a.np / 8; o += blockDim.x)
+        reinterpret_cast<uint4*>(a.gperm + (size_t)nxt * a.np)[o] = __ldcg(src + o);
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        a.gkey[nxt] = k;
+        a.counter[1] = 0u;
+        a.counter[2] = 0u;
+        a.fkey[0] = a.fkey[1] = ULLONG_MAX;
+        __threadfence();
+        asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(a.counter + 3), "r"((uint32_t)done) : "memory");
+    }
+}
+
+template <int NP>
+__device__ __forceinline__ void dg_stage_fast(const DgArgs& a, uint16_t* g_sm, int64_t t, int64_t t0,
+                                              unsigned long long* s_gk, int per_cta) {
+    __syncthreads();
+    if (threadIdx.x < 32) {
+        unsigned long long k = 0;
+        if (threadIdx.x == 0) {
+            if (t > t0) {
+                const unsigned int target = dg_target(t, t0);
+                while (dg_acquire(a.counter + 1 + (int)(t & 1)) < target) {
+                }
+            }
+            k = __ldcg((t > t0 ? a.fkey : a.gkey) + (t & 1));
+            if (t > t0 && blockIdx.x == 0 && a.trace) a.trace[t] = (int64_t)(k >> 32);  // line 5 of iteration t
+        }
+        k = __shfl_sync(kFull, k, 0);
+        if (k != *s_gk) {  // the swarm best row changes only with its key
+            const int16_t* src = t > t0 ? a.slots + ((size_t)(t & 1) * gridDim.x + dg_cta_of(a, k, per_cta)) * a.np
+                                        : a.gperm + (size_t)(t & 1) * a.np;
+            for (int o = 8 * (int)threadIdx.x; o < NP; o += 256)
+                *reinterpret_cast<uint4*>(g_sm + o) = __ldcg(reinterpret_cast<const uint4*>(src + o));
+            __syncwarp();
+            if (threadIdx.x == 0) *s_gk = k;
+        }
     }
     __syncthreads();
 }
@@ -405,7 +523,7 @@ __global__ void __launch_bounds__(DgSmem<DG, E, UCD>::THREADS) dpsog_init_kernel
         wkey = key < wkey ? key : wkey;
         __syncwarp();
     }
-    dg_publish<S::W>(a, wkey, 0, 1, false, 0u, false);
+    dg_publish<S::W>(a, wkey, 0, 1, false, 0u, false, true);
 }
 
 // ---- warp-wide crossovers (one particle at a time, all 32 lanes): a crossover is applied with
@@ -518,6 +636,16 @@ __global__ void __launch_bounds__(DgSmem<DG, E, UCD>::THREADS, 1) dpsog_iter_ker
             }
     const double u2 = 2.3283064365386962890625e-10;
     uint16_t* g_sm = reinterpret_cast<uint16_t*>(smem + S::G_OFF);
+    __shared__ unsigned long long s_gk;  // key of the swarm best row held in g_sm
+    __shared__ unsigned long long s_slot[2];  // keys of this CTA's slot rows (single-GPU publish)
+    if (threadIdx.x == 0) s_gk = s_slot[0] = s_slot[1] = ULLONG_MAX;
+    const bool fast = a.pw <= 1;
+    auto stage = [&](int64_t t) {
+        if (fast)
+            dg_stage_fast<NP>(a, g_sm, t, t0, &s_gk, per_cta);
+        else
+            dg_cta_stage<NP>(a, g_sm, (uint32_t)t, &s_gk);
+    };
     // swarm best at line 5 of iteration t0 (after a host-side exchange when stepping across GPUs)
     if (a.trace && blockIdx.x == 0 && threadIdx.x == 0) a.trace[t0] = (int64_t)(a.gkey[t0 & 1] >> 32);
     for (int64_t t = t0; t < t1; ++t) {
@@ -573,7 +701,7 @@ __global__ void __launch_bounds__(DgSmem<DG, E, UCD>::THREADS, 1) dpsog_iter_ker
             // everything below needs the swarm best of iteration t (F3) or writes the personal
             // best the last CTA of the previous publish may still be copying
             if (!have_g) {
-                dg_cta_stage<NP>(a, g_sm, (uint32_t)t);
+                stage(t);
                 have_g = true;
             }
 #pragma unroll
@@ -621,9 +749,12 @@ __global__ void __launch_bounds__(DgSmem<DG, E, UCD>::THREADS, 1) dpsog_iter_ker
         }
         // a warp without particles never waited: the previous publish must be complete before
         // this one re-uses its key slot and counter
-        if (!have_g) dg_cta_stage<NP>(a, g_sm, (uint32_t)t);
+        if (!have_g) stage(t);
         // line 5 (iteration t+1): swarm best (traced here when iteration t+1 runs in this launch)
-        dg_publish<S::W>(a, wkey, nxt, cur, true, (uint32_t)(t + 1), t + 1 < t1);
+        if (fast)
+            dg_publish_fast<S::W>(a, wkey, nxt, t + 1, t0, t + 1 == t1, s_slot, per_cta);
+        else
+            dg_publish<S::W>(a, wkey, nxt, cur, true, (uint32_t)(t + 1), t + 1 < t1, t + 1 == t1);
     }
 }
 
@@ -665,6 +796,7 @@ template <int DG, int E, bool UCD>
 cudaError_t dg_begin(const Instance& I, const DgArgs& a, int64_t particles, cudaStream_t s) {
     cudaError_t e = cudaMemsetAsync(a.gkey, 0xff, 2 * sizeof(unsigned long long), s);
     if (e == cudaSuccess) e = cudaMemsetAsync(a.counter, 0, 4 * sizeof(unsigned int), s);
+    if (e == cudaSuccess) e = cudaMemsetAsync(a.fkey, 0xff, 2 * sizeof(unsigned long long), s);
     if (e != cudaSuccess) return e;
     const DgShape sh = dg_shape<DG, E, UCD>(I, dpsog_init_kernel<DG, E, UCD>, particles);
     dpsog_init_kernel<DG, E, UCD><<<sh.blocks, sh.warps * 32, sh.smem, s>>>(a);
@@ -750,7 +882,8 @@ static DgArgs dg_args(const Instance& I, const DpsoLaunch& p, const DpsoWsPtrs& 
     a.gkey = w.gkey;
     a.gperm = w.gperm;
     a.counter = w.counter;
-    a.ctakeys = w.ctakeys;
+    a.slots = w.slots;
+    a.fkey = reinterpret_cast<unsigned long long*>(w.counter + 4);
     a.err = I.err;
     if (p.peer && I.peer && I.peer->open) {
         a.pw = I.peer->world;

@@ -143,7 +143,7 @@ struct DpsoWsPtrs {
     unsigned long long* gkey;
     int16_t* gperm;
     unsigned int* counter;
-    unsigned long long* ctakeys;  // per-CTA minimum keys (group layout's publish), kDpsoMaxCtas
+    int16_t* slots;  // [2][kDpsoMaxCtas or fewer][np]: each CTA's best personal-best row (group publish)
     int np;
 };
 constexpr int kDpsoMaxCtas = 8192;

@@ -147,7 +147,7 @@ def main():
         dt = timed(lambda r=0: cdd.cdd_eval_batch(iw, pw[r & 1], ow), reps=5)
         out("G", f"generic cdd_eval_batch n={nw} (p<=1000, alpha,beta<=1e4), {batch} sequences", batch / dt,
             "evals/s", batch * (2 * nw + 8) / dt / 1e9, hbm, "GB/s",
-            "int64 arithmetic, int4 record gathers from L1/L2 (3 passes)")
+            "int64 arithmetic, int4 record gathers from L1/L2 (one pass)")
         if nw == 1000:
             C, S = 16384, 200
             ws = cdd.sa_run(iw, C, S, seed=1, T0=1e9)["workspace"]
