@@ -126,6 +126,8 @@ __global__ void __launch_bounds__(kSchedWarps * 32, CDD_SCHED_MINB) schedule_ker
     int32_t* myX = X_s + lane * CS;
     const int64_t warps = (int64_t)gridDim.x * kSchedWarps;
     bool bad = false;
+    uint32_t vmax = 0;                 // u16x2 maximum of the ids of whole vector chunks
+    const uint32_t NN = N | (N << 16);
     // pairs of positions per store when rows of C (and X) are 16-byte aligned
     const bool pairs = E >= 2 && n % 2 == 0 && (reinterpret_cast<uintptr_t>(a.C) & 15u) == 0 &&
                        (!UCD || (reinterpret_cast<uintptr_t>(a.X) & 7u) == 0);
@@ -156,20 +158,29 @@ __global__ void __launch_bounds__(kSchedWarps * 32, CDD_SCHED_MINB) schedule_ker
                     const uint32_t w[4] = {(uint32_t)pre[t].x, (uint32_t)pre[t].y, (uint32_t)pre[t].z,
                                            (uint32_t)pre[t].w};
                     uint32_t o[4];
+                    if (8 * c + 8 <= n) {
+                        // whole chunk inside the row: the maximum id (as u16: negative ids are
+                        // >= 32768) raises the flag at the end; out-of-range ids read the sentinel's
+                        // zero record (the row's results are unspecified, P:29-33 ids are 0..n-1)
+                        vmax = __vimax3_u16x2(__vimax3_u16x2(vmax, w[0], w[1]), w[2], w[3]);
 #pragma unroll
-                    for (int h = 0; h < 4; ++h) {
-                        uint32_t id2[2] = {w[h] & 0xffffu, w[h] >> 16};
+                        for (int h = 0; h < 4; ++h) o[h] = __vminu2(w[h], NN);
+                    } else {
 #pragma unroll
-                        for (int u = 0; u < 2; ++u) {
-                            const int k = 8 * c + 2 * h + u;
-                            if (k >= n) {
-                                id2[u] = N;  // the caller's padding: sentinel
-                            } else if (id2[u] >= N) {  // an id outside [0, n) (incl. negative)
-                                bad = true;
-                                id2[u] = 0u;
+                        for (int h = 0; h < 4; ++h) {
+                            uint32_t id2[2] = {w[h] & 0xffffu, w[h] >> 16};
+#pragma unroll
+                            for (int u = 0; u < 2; ++u) {
+                                const int k = 8 * c + 2 * h + u;
+                                if (k >= n) {
+                                    id2[u] = N;  // the caller's padding: sentinel
+                                } else if (id2[u] >= N) {  // an id outside [0, n) (incl. negative)
+                                    bad = true;
+                                    id2[u] = 0u;
+                                }
                             }
+                            o[h] = id2[0] | (id2[1] << 16);
                         }
-                        o[h] = id2[0] | (id2[1] << 16);
                     }
                     const int k = 8 * c;
                     *reinterpret_cast<uint4*>(ids_s + (k >> lE) * IS + (k & (E - 1))) =
@@ -309,9 +320,17 @@ __global__ void __launch_bounds__(kSchedWarps * 32, CDD_SCHED_MINB) schedule_ker
         int64_t* Crow = a.C + row * (int64_t)n;
         const int64_t cb = UCD ? a.d : st;
         if (pairs) {  // 16-byte streaming stores of position pairs (same lane segment: E even)
-            for (int k = 2 * lane; k < n; k += 64) {
-                const int idx = (k >> lE) * CS + (k & (E - 1));
-                __stcs(reinterpret_cast<longlong2*>(Crow + k), make_longlong2(cb + C_s[idx], cb + C_s[idx + 1]));
+            if constexpr (E <= 64) {
+                // 64 positions per step = 64/E whole segments: the staged index advances by a constant
+                int idx = ((2 * lane) >> lE) * CS + ((2 * lane) & (E - 1));
+                longlong2* dst = reinterpret_cast<longlong2*>(Crow) + lane;
+                for (int k = 2 * lane; k < n; k += 64, idx += (64 / E) * CS, dst += 32)
+                    __stcs(dst, make_longlong2(cb + C_s[idx], cb + C_s[idx + 1]));
+            } else {
+                for (int k = 2 * lane; k < n; k += 64) {
+                    const int idx = (k >> lE) * CS + (k & (E - 1));
+                    __stcs(reinterpret_cast<longlong2*>(Crow + k), make_longlong2(cb + C_s[idx], cb + C_s[idx + 1]));
+                }
             }
         } else {
             for (int k = lane; k < n; k += 32) Crow[k] = cb + C_s[(k >> lE) * CS + (k & (E - 1))];
@@ -329,7 +348,7 @@ __global__ void __launch_bounds__(kSchedWarps * 32, CDD_SCHED_MINB) schedule_ker
         }
         __syncwarp();
     }
-    if (bad) atomicOr(a.err, 1);
+    if (bad || (vmax & 0xffffu) >= N || (vmax >> 16) >= N) atomicOr(a.err, 1);
 }
 
 }  // namespace

@@ -85,6 +85,10 @@ def main():
         dt = timed(lambda r=0: cdd.cdd_schedule_batch(ic, sp), reps=5)
         out("F1", f"cdd_schedule_batch n={n}, 2^17 sequences", B / dt, "schedules/s",
             B * (2 * n + 8 * n + 16) / dt / 1e9, hbm, "GB/s", "C int64 [B, n] written + start + penalty")
+        dt = timed(lambda r=0: cdd.cdd_schedule_batch(iu, sp, "ucddcp"), reps=5)
+        out("F1", f"ucddcp schedule_batch n={n}, 2^17 sequences", B / dt, "schedules/s",
+            B * (2 * n + 12 * n + 16) / dt / 1e9, hbm, "GB/s",
+            "C int64 + X int32 [B, n] written + start + penalty")
 
     # A8 T0
     T0 = 5000
