@@ -53,8 +53,8 @@ __device__ __forceinline__ int64_t warp_sum64(int64_t v) {
     return v;
 }
 
-// Shared-memory layout (dynamic): the instance tables by job id (ab u32, p u8 [, M u8, X u8,
-// gamma u16], each array padded to 16 bytes), then per warp: the sequence's ids in lane segments
+// Shared-memory layout (dynamic): the instance tables by job id (ab u32, p u8 [, M | X << 8 |
+// gamma << 16 u32], each array padded to 16 bytes), then per warp: the sequence's ids in lane segments
 // of E positions (E = pow2 >= ceil(n/32), segments padded by 16 bytes), and the output staging
 // C [and X] (int32) in lane segments padded by one element, so that the lane-contiguous compute
 // writes and the coalesced copy-out reads are both (nearly) conflict free.  C is staged relative
@@ -72,7 +72,7 @@ __host__ __device__ inline SchedLayout sched_layout(int n, bool ucd, int warps) 
     while ((32 << L.lE) < n) ++L.lE;
     L.E = 1 << L.lE;
     const uint32_t N = (uint32_t)n;
-    L.tab_bytes = al16(4 * (N + 1)) + al16(N + 1) + (ucd ? al16(N + 1) + al16(N + 1) + al16(2 * (N + 1)) : 0u);
+    L.tab_bytes = al16(4 * (N + 1)) + al16(N + 1) + (ucd ? al16(4 * (N + 1)) : 0u);
     L.ids_off = 0;
     L.c_off = al16(32u * (2u * L.E + 16u));
     L.x_off = L.c_off + al16(32u * 4u * (L.E + 1u));
@@ -99,18 +99,14 @@ __global__ void __launch_bounds__(kSchedWarps * 32, CDD_SCHED_MINB) schedule_ker
     // is 0 -- they repeat C_{n-1}, so no slot needs an index test)
     uint32_t* t_ab = reinterpret_cast<uint32_t*>(smem);
     uint8_t* t_p = smem + al16(4 * (N + 1));
-    uint8_t* t_m = t_p + al16(N + 1);
-    uint8_t* t_x = t_m + al16(N + 1);
-    uint16_t* t_g = reinterpret_cast<uint16_t*>(t_x + al16(N + 1));
+    uint32_t* t_mxg = reinterpret_cast<uint32_t*>(t_p + al16(N + 1));  // UCDDCP: M | X << 8 | gamma << 16
     for (int j = threadIdx.x; j <= n; j += blockDim.x) {
         const bool v = j < n;
         t_ab[j] = v ? __ldg(a.ab + j) : 0u;
         t_p[j] = v ? __ldg(a.p + j) : (uint8_t)0;
-        if constexpr (UCD) {
-            t_m[j] = v ? __ldg(a.m + j) : (uint8_t)0;
-            t_x[j] = v ? __ldg(a.x + j) : (uint8_t)0;
-            t_g[j] = v ? __ldg(a.g + j) : (uint16_t)0;
-        }
+        if constexpr (UCD)
+            t_mxg[j] = v ? (uint32_t)__ldg(a.m + j) | ((uint32_t)__ldg(a.x + j) << 8) | ((uint32_t)__ldg(a.g + j) << 16)
+                         : 0u;
     }
     uint8_t* wbase = smem + Ly.tab_bytes + (size_t)wib * Ly.warp_bytes;
     uint16_t* ids_s = reinterpret_cast<uint16_t*>(wbase + Ly.ids_off);
@@ -199,33 +195,29 @@ __global__ void __launch_bounds__(kSchedWarps * 32, CDD_SCHED_MINB) schedule_ker
             }
             __syncwarp();
         }
-        // lane totals, then exclusive bases; the records stay in registers for the later passes
-        // (the compiler cannot keep them across the shared-memory stores of C otherwise)
-        // (CDD only: the UCDDCP passes need more per-position data than the registers hold)
-        constexpr int RC = UCD ? 1 : E;
-        uint32_t rr[RC], pq[(RC + 3) / 4];
+        // lane totals, then exclusive bases; the alpha|beta records stay in registers for the later
+        // passes (the compiler cannot keep them across the shared-memory stores of C otherwise)
+        constexpr int PQ = UCD ? 1 : (E + 3) / 4;
+        uint32_t rr[E], pq[PQ];
         #pragma unroll
-        for (int i = 0; i < (RC + 3) / 4; ++i) pq[i] = 0u;
+        for (int i = 0; i < PQ; ++i) pq[i] = 0u;
         int32_t tP = 0, tA = 0, tB = 0;
         #pragma unroll
         for (int i = 0; i < E; ++i) {
             const int j = myids[i];
             const uint32_t r = t_ab[j];
-            const uint32_t pj = t_p[j];
+            rr[i] = r;
             if constexpr (!UCD) {
-                rr[i] = r;
+                const uint32_t pj = t_p[j];
                 pq[i / 4] |= pj << (8 * (i % 4));
+                tP += (int32_t)pj;
             }
-            tP += (int32_t)pj;
             tA += (int32_t)(r & 0xffffu);
             tB += (int32_t)(r >> 16);
         }
-        auto rec_r = [&](int i) {
-            if constexpr (UCD) return t_ab[myids[i]];
-            else return rr[i];
-        };
+        auto rec_r = [&](int i) { return rr[i]; };
         auto rec_p = [&](int i) {
-            if constexpr (UCD) return (int32_t)t_p[myids[i]];
+            if constexpr (UCD) return 0;  // (C_{k0} is the CDD's; the UCDDCP uses the prefix of p')
             else return (int32_t)((pq[i / 4] >> (8 * (i % 4))) & 0xffu);
         };
         const int32_t Pb = warp_excl_scan(tP, lane), Ab = warp_excl_scan(tA, lane),
@@ -267,48 +259,43 @@ __global__ void __launch_bounds__(kSchedWarps * 32, CDD_SCHED_MINB) schedule_ker
                 pen += (int64_t)(r & 0xffffu) * max(0, Dl - c) + (int64_t)(r >> 16) * max(0, c - Dl);
             }
         } else {
-            // compression decisions and the lane totals of p'
-            int32_t tQ = 0;
+            // compression decisions (Property 2: X_k = P_k - M_k iff the weight of position k
+            // exceeds gamma_k), p' = P - X_k staged next to X, the lane totals of p', the prefix
+            // of p' through k0 on its lane, and the gamma part of the penalty
+            int32_t tQ = 0, qk = 0, pg = 0;  // pg <= E * 255 * 65535 < 2^31
             {
                 int32_t A = Ab, B = Bb;  // exclusive prefixes
                 #pragma unroll
-        for (int i = 0; i < E; ++i) {
-                    const int j = myids[i];
-                    const uint32_t r = t_ab[j];
-                    const int32_t w = k_lo + i <= k0 ? A : Btot - B;
-                    const int32_t xk = w > (int32_t)t_g[j] ? (int32_t)t_x[j] : 0;
-                    myX[i] = xk;
-                    tQ += (int32_t)t_m[j] + (int32_t)t_x[j] - xk;
+                for (int i = 0; i < E; ++i) {
+                    const uint32_t r = rr[i];
+                    const uint32_t mxg = t_mxg[myids[i]];
+                    const int32_t g = (int32_t)(mxg >> 16), xj = (int32_t)((mxg >> 8) & 0xffu);
+                    const bool early = k_lo + i <= k0;
+                    const int32_t w = early ? A : Btot - B;
+                    const int32_t xk = w > g ? xj : 0;
+                    const int32_t q = (int32_t)(mxg & 0xffu) + xj - xk;
+                    reinterpret_cast<uint32_t*>(myX)[i] = (uint32_t)xk | ((uint32_t)q << 16);
+                    tQ += q;
+                    qk += early ? q : 0;
+                    pg += g * xk;
                     A += (int32_t)(r & 0xffffu);
                     B += (int32_t)(r >> 16);
                 }
             }
             const int32_t Qb = warp_excl_scan(tQ, lane);
-            // C'_{k0}: inclusive prefix of p' at k0
-            int32_t Qk0 = 0;
-            {
-                int32_t q = Qb;
-                #pragma unroll
-        for (int i = 0; i < E; ++i) {
-                    const int j = myids[i];
-                    q += (int32_t)t_m[j] + (int32_t)t_x[j] - myX[i];
-                    if (k_lo + i == k0) Qk0 = q;
-                }
-            }
-            Qk0 = __shfl_sync(kFull, Qk0, owner);
+            // C'_{k0}: inclusive prefix of p' at k0 (on the lane holding k0)
+            const int32_t Qk0 = __shfl_sync(kFull, Qb + qk, owner);
             st = a.d - Qk0;
             int32_t q = Qb;
             #pragma unroll
-        for (int i = 0; i < E; ++i) {
-                const int j = myids[i];
-                const uint32_t r = t_ab[j];
-                const int32_t xk = myX[i];
-                q += (int32_t)t_m[j] + (int32_t)t_x[j] - xk;
+            for (int i = 0; i < E; ++i) {
+                const uint32_t r = rr[i];
+                q += (int32_t)(reinterpret_cast<const uint32_t*>(myX)[i] >> 16);
                 const int32_t c = q - Qk0;  // C_k - d
                 myC[i] = c;
-                pen += (int64_t)(r & 0xffffu) * max(0, -c) + (int64_t)(r >> 16) * max(0, c) +
-                       (int64_t)t_g[j] * xk;
+                pen += (int64_t)(r & 0xffffu) * max(0, -c) + (int64_t)(r >> 16) * max(0, c);
             }
+            pen += pg;
         }
         pen = warp_sum64(pen);
         if (lane == 0) {
@@ -340,10 +327,10 @@ __global__ void __launch_bounds__(kSchedWarps * 32, CDD_SCHED_MINB) schedule_ker
             if (pairs) {
                 for (int k = 2 * lane; k < n; k += 64) {
                     const int idx = (k >> lE) * CS + (k & (E - 1));
-                    __stcs(reinterpret_cast<int2*>(Xrow + k), make_int2(X_s[idx], X_s[idx + 1]));
+                    __stcs(reinterpret_cast<int2*>(Xrow + k), make_int2(X_s[idx] & 0xffff, X_s[idx + 1] & 0xffff));
                 }
             } else {
-                for (int k = lane; k < n; k += 32) Xrow[k] = X_s[(k >> lE) * CS + (k & (E - 1))];
+                for (int k = lane; k < n; k += 32) Xrow[k] = X_s[(k >> lE) * CS + (k & (E - 1))] & 0xffff;
             }
         }
         __syncwarp();
