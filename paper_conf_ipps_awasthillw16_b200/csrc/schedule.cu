@@ -86,7 +86,7 @@ constexpr int kSchedWarps = 4;
 #endif
 
 template <bool UCD, int E>
-__global__ void __launch_bounds__(kSchedWarps * 32, CDD_SCHED_MINB) schedule_kernel(SchedArgs a) {
+__global__ void __launch_bounds__(kSchedWarps * 32, UCD ? 3 : CDD_SCHED_MINB) schedule_kernel(SchedArgs a) {
     extern __shared__ __align__(16) uint8_t smem[];
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
     const int n = a.n;
