@@ -908,6 +908,8 @@ Grid sag_grid(const Instance& I, int64_t chains) {
     int sms = 148, occ = 1;
     resident_ctas(reinterpret_cast<const void*>(sa_group_kernel<G, E, UCD, TRACE, MV>), I.device, kGThreads, gr.smem,
                   &sms, &occ);
+    // CDD_SA_OCC=k: at most k CTAs per SM (occupancy experiments)
+    if (const char* v = getenv("CDD_SA_OCC")) occ = std::max(1, std::min(occ, atoi(v)));
     const int64_t need = (chains + CPB - 1) / CPB;
     const int64_t cap = (int64_t)sms * occ;
     gr.blocks = (int)(need < cap ? (need < 1 ? 1 : need) : cap);

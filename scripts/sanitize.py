@@ -44,5 +44,32 @@ cdd.dpso_peer_reset(ins)
 cdd.SaSync(ins, 1024, 3, 2, seed=3, t0_samples=100).run_peer()
 cdd.dpso_peer_destroy(ins)
 cdd.cdd_check(ins)
+# the insertion and window moves (R11b, R11c)
+ins = cdd.Instance.from_gen(gen.cdd_instance(1000, 3, 0.4))
+for mv in ("insert", "window"):
+    cdd.sa_run(ins, 256, 30, seed=5, t0_samples=100, move=mv)
+    cdd.sa_run(ins, 40, 30, seed=5, t0_samples=100, move=mv, lanes=32)
+cdd.cdd_check(ins)
+# the generic path (values outside the packed ranges; n up to 32767)
+import numpy as np  # noqa: E402
+
+rng = np.random.default_rng(7)
+for nw in (300, 1500, 5000):
+    P = rng.integers(1, 1001, nw).astype(np.int32)
+    a = rng.integers(1, 10001, nw).astype(np.int32)
+    b = rng.integers(1, 10001, nw).astype(np.int32)
+    M = (P - rng.integers(0, P)).astype(np.int32)
+    g = rng.integers(1, 10001, nw).astype(np.int32)
+    for d in (int(0.4 * int(P.sum())), int(P.sum()) + 3):
+        iw = cdd.Instance(P, a, b, d, M, g)
+        pw = gen.random_perms_device(40, nw, 9, ld=nw)
+        cdd.cdd_eval_batch(iw, pw)
+        cdd.cdd_schedule_batch(iw, pw[:8])
+        if d > int(P.sum()):
+            cdd.ucddcp_eval_batch(iw, pw)
+            cdd.cdd_schedule_batch(iw, pw[:8], "ucddcp")
+        if nw <= 1500:
+            cdd.sa_run(iw, 64, 10, seed=6, t0_samples=50, move="insert" if nw == 300 else "pert_fy")
+        cdd.cdd_check(iw)
 torch.cuda.synchronize()
 print("sanitize run ok")
