@@ -641,6 +641,19 @@ def bench_quality(lib, dev, stream):
             per_h[f"{h:.1f}"].append(gap(g, lib.best_get(ins)[0]))
     out["config5"] = summary(sum(per_h.values(), []), per_h={k: summary(v)["mean_gap_pct"] for k, v in per_h.items()},
                              workload=f"CDD n=1000, 10 instances x 4 h, SA {CHAINS} chains x {SA_STEPS} steps")
+    # the other neighbourhoods on the same 40 instances (R11b insertion, R11c contiguous window of
+    # Pert = 4 positions; swap) beside the paper's Pert-FY reading R11 above
+    moves = {}
+    for mv in ("window", "swap", "insert"):
+        rows = []
+        for k in range(1, 11):
+            for h in HS:
+                g = gen.cdd_instance(N_JOBS, k, h)
+                ins = lib.Instance.from_gen(g, device=dev.index)
+                lib.sa_run(ins, CHAINS, SA_STEPS, seed=RUN_SEED, t0_samples=T0_SAMPLES, move=mv)
+                rows.append(gap(g, lib.best_get(ins)[0]))
+        moves[mv] = summary(rows)
+    out["config5"]["moves"] = moves
     out["seconds"] = time.time() - t0
     out["reference"] = ("% gap to tests/golden/best_known.json (best of long GPU searches, every penalty "
                         "re-evaluated by the oracle); the paper's Table II reports %Delta to [7]'s results "

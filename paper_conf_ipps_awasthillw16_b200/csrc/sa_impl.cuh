@@ -430,6 +430,78 @@ __device__ __forceinline__ uint2 rot8(uint2 A, uint32_t nb, bool left, uint32_t 
     return R;
 }
 
+// CDD byte rows in chunks of 16 positions (one 16-byte word per row; E a multiple of 16): half
+// the rounds of the 8-position chunks, and chunks wholly inside the range skip the masks.
+__device__ __forceinline__ uint32_t rot_mask16(int c, int lo, int hi, bool left) {
+    const int a = max((left ? lo : lo + 1) - c, 0), b = min((left ? hi : hi + 1) - c, 16);
+    return a < b ? ((b >= 32 ? 0xffffffffu : (1u << b) - 1u) & ~((1u << a) - 1u)) : 0u;
+}
+__device__ __forceinline__ uint4 rot_b16(uint4 A, uint32_t nb, bool left, uint32_t m16) {
+    uint4 S;
+    if (left) {
+        S.x = __funnelshift_r(A.x, A.y, 8);
+        S.y = __funnelshift_r(A.y, A.z, 8);
+        S.z = __funnelshift_r(A.z, A.w, 8);
+        S.w = __funnelshift_r(A.w, nb, 8);
+    } else {
+        S.x = __funnelshift_l(nb << 24, A.x, 8);
+        S.y = __funnelshift_l(A.x, A.y, 8);
+        S.z = __funnelshift_l(A.y, A.z, 8);
+        S.w = __funnelshift_l(A.z, A.w, 8);
+    }
+    if (m16 == 0xffffu) return S;
+    const uint32_t b0 = byte_mask(m16 & 15u), b1 = byte_mask((m16 >> 4) & 15u), b2 = byte_mask((m16 >> 8) & 15u),
+                   b3 = byte_mask(m16 >> 12);
+    return make_uint4((S.x & b0) | (A.x & ~b0), (S.y & b1) | (A.y & ~b1), (S.z & b2) | (A.z & ~b2),
+                      (S.w & b3) | (A.w & ~b3));
+}
+template <int G, int E>
+__device__ __forceinline__ void group_rotate_rows16(const GChain<G, E, false>& ch, int lo, int hi, bool left,
+                                                    bool act, int l) {
+    using C = GChain<G, E, false>;
+    static_assert(E % 16 == 0, "16-position chunks stay inside a lane row");
+    const int c0 = lo & ~15, c1 = hi & ~15;
+    const int nch = act && hi > lo ? (c1 - c0) / 16 + 1 : 0;
+    const int rounds = (int)__reduce_max_sync(kFull, (uint32_t)((nch + G - 1) / G));
+    const int wsrc = left ? lo : hi;
+    uint2 wv = make_uint2(0u, 0u);
+    if (l == 0 && nch) wv = pos_read<G, E, false>(ch, wsrc);
+    for (int r = 0; r < rounds; ++r) {
+        const int j = r * G + l;
+        const bool v = j < nch;
+        const int c = left ? c0 + 16 * j : c1 - 16 * j;
+        const uint32_t m16 = v ? rot_mask16(c, lo, hi, left) : 0u;
+        const bool nbv = left ? ((m16 >> 15) & 1u) : (m16 & 1u);
+        const int kn = left ? c + 16 : c - 1;
+        uint4 Ra = make_uint4(0, 0, 0, 0), Rb = Ra, Rp = Ra;
+        if (v) {
+            const int i = C::rb(c), in = C::rb(kn);
+            Ra = *reinterpret_cast<const uint4*>(ch.a8() + i);
+            Rb = *reinterpret_cast<const uint4*>(ch.b8() + i);
+            Rp = *reinterpret_cast<const uint4*>(ch.pb() + i);
+            uint32_t na = 0u, nb = 0u, np = 0u;
+            if (nbv) {
+                na = ch.a8()[in];
+                nb = ch.b8()[in];
+                np = ch.pb()[in];
+            }
+            Ra = rot_b16(Ra, na, left, m16);
+            Rb = rot_b16(Rb, nb, left, m16);
+            Rp = rot_b16(Rp, np, left, m16);
+        }
+        __syncwarp();
+        if (v && m16) {
+            const int i = C::rb(c);
+            *reinterpret_cast<uint4*>(ch.a8() + i) = Ra;
+            *reinterpret_cast<uint4*>(ch.b8() + i) = Rb;
+            *reinterpret_cast<uint4*>(ch.pb() + i) = Rp;
+        }
+        __syncwarp();
+    }
+    if (l == 0 && nch) pos_write<G, E, false>(ch, left ? hi : lo, wv);
+    __syncwarp();
+}
+
 // Rotates the records (IDS = false: ab, p / M, X, gamma in shared memory) or the job ids of the
 // group's current slot (IDS = true, global) over [lo, hi].  act: this group has a move (the other
 // groups of the warp run the same number of rounds with nothing to do).
@@ -437,6 +509,10 @@ template <int G, int E, bool UCD, bool IDS>
 __device__ __forceinline__ void group_rotate(const GChain<G, E, UCD>& ch, int16_t* ids, int lo, int hi,
                                              bool left, bool act, int l) {
     using C = GChain<G, E, UCD>;
+    if constexpr (!IDS && !UCD && E % 16 == 0) {
+        group_rotate_rows16<G, E>(ch, lo, hi, left, act, l);
+        return;
+    }
     const int c0 = lo & ~7, c1 = hi & ~7;
     const int nch = act && hi > lo ? (c1 - c0) / 8 + 1 : 0;
     const int rounds = (int)__reduce_max_sync(kFull, (uint32_t)((nch + G - 1) / G));

@@ -17,7 +17,7 @@ $N -k regex:eval2 -s 1 -c 1 -o p_ev python ../$S/eval_sweep.py --reps 2 1000 > /
 $N -k regex:eval2 -s 1 -c 1 -o p_evu python ../$S/eval_sweep.py --problem ucddcp --reps 2 1000 > /dev/null 2>&1
 $N -k regex:dpsog_iter -c 1 -o p_dp python ../$S/dpso_time.py 500 > /dev/null 2>&1
 $N -k regex:schedule -s 1 -c 1 -o p_sch python ../$S/row_bench.py F1 > /dev/null 2>&1
-$N -k "regex:schedule_kernel<true" -s 1 -c 1 -o p_schu python ../$S/row_bench.py F1 > /dev/null 2>&1
+$N --kernel-name-base demangled -k "regex:schedule_kernel<.bool.1" -s 1 -c 1 -o p_schu python ../$S/row_bench.py F1 > /dev/null 2>&1
 { python ../$S/ncu_summary.py p_sa.ncu-rep 327745536; echo; python ../$S/ncu_stalls.py p_sa.ncu-rep 25; echo; python ../$S/ncu_lines.py p_sa.ncu-rep 327745536 40; } > r2_ncu_sa_full.txt 2>&1
 { python ../$S/ncu_summary.py p_ev.ncu-rep 1048576; echo; python ../$S/ncu_stalls.py p_ev.ncu-rep 25; echo; python ../$S/ncu_lines.py p_ev.ncu-rep 1048576 40; } > r2_ncu_eval2_cdd_full.txt 2>&1
 { python ../$S/ncu_summary.py p_evu.ncu-rep 1048576; echo; python ../$S/ncu_stalls.py p_evu.ncu-rep 25; echo; python ../$S/ncu_lines.py p_evu.ncu-rep 1048576 40; } > r2_ncu_eval2_ucddcp_full.txt 2>&1

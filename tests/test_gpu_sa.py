@@ -1,4 +1,6 @@
 """GPU parity: T0 rule and SA chains replayed step by step against the oracle (bit-exact)."""
+import os
+
 import numpy as np
 import pytest
 
@@ -318,17 +320,38 @@ def test_bench_config_sampled_parity(lib):
     ins = lib.Instance.from_gen(inst)
     T0 = lib.sa_t0(ins, "cdd", seed=bench.RUN_SEED, samples=bench.T0_SAMPLES)
     res = lib.sa_run(ins, bench.CHAINS, bench.SA_STEPS, seed=bench.RUN_SEED, T0_dev=T0,
-                     chain_best=True)
+                     chain_best=True, chain_final=True)
     torch.cuda.synchronize()
     pen, perm, gid = lib.best_get(ins)
     cb = res["chain_best"].cpu().numpy()
+    cf = res["chain_final"].cpu().numpy()
     pr = _prob(inst)
     assert oracle.cdd_eval(pr, perm) == pen == cb.min() and gid == int(np.argmin(cb))
     T0v = float(T0.item())
     assert T0v == oracle.t0(pr, oracle.CDD, bench.RUN_SEED, bench.T0_SAMPLES)
     p = oracle.sa_params(chains=1, steps=bench.SA_STEPS, seed=bench.RUN_SEED)
-    for c in [0, 1, 31, 4096, 40000, bench.CHAINS - 1, gid]:
-        assert oracle.sa_chain(pr, p, T0v, c)["E_best"] == cb[c], c
+    # 1024 sampled chains (edges of warps, CTAs and rounds, the winner, the rest seeded-random),
+    # replayed by the oracle on the host threads (ctypes releases the GIL)
+    rng = np.random.default_rng(5)
+    sample = sorted(set([0, 1, 3, 4, 31, 32, 4096, 40000, bench.CHAINS - 1, gid] +
+                        rng.choice(bench.CHAINS, 1014, replace=False).tolist()))
+    got = {}
+
+    def work(cs):
+        for c in cs:
+            r = oracle.sa_chain(pr, p, T0v, c)
+            got[c] = (r["E_best"], r["E_final"])
+
+    import threading
+
+    nt = max(1, min(16, os.cpu_count() or 1))
+    ts = [threading.Thread(target=work, args=(sample[i::nt],)) for i in range(nt)]
+    for t in ts:
+        t.start()
+    for t in ts:
+        t.join()
+    for c in sample:
+        assert got[c] == (cb[c], cf[c]), c
 
 
 def test_configs_2_3_sampled_parity(lib):
