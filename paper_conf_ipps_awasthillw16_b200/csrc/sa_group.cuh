@@ -282,17 +282,25 @@ __device__ __forceinline__ int32_t boundary_two_level(const GChain<G, E>& ch, in
         return gscan<G>(tot) - tot + __shfl_sync(kFull, ex, blk, G);  // row-relative start
     };
     uint32_t v[L2];
-    uint32_t run = spread(own, v), cinc = 0;
-    const bool first_sat = run <= key;
+    uint32_t run;
+    // D - C at the row start.  C_{k0} matters only when the boundary row is k0's (Ls == Lk); when
+    // d's row comes first (Lt < Lk), C_{k0} > d and D = d -- the usual case for restrictive due
+    // dates -- so a warp whose chains all have Ls < Lk skips the search for C_{k0}
+    int32_t Dr = d - PbS;
+    if (__any_sync(kFull, Ls == Lk)) {
+        run = spread(own, v);
+        uint32_t cinc = 0;
+        const bool first_sat = run <= key;
 #pragma unroll
-    for (int i = 0; i < L2; ++i) {
-        const bool sat = run <= key;
-        run += v[i];
-        cinc = sat ? run : cinc;
+        for (int i = 0; i < L2; ++i) {
+            const bool sat = run <= key;
+            run += v[i];
+            cinc = sat ? run : cinc;
+        }
+        const int own2 = max(0, hibit(group_ballot<G>(first_sat, gbase)));
+        const int32_t Ck0 = PbS + (int32_t)(__shfl_sync(kFull, cinc, own2, G) & 0xffffu);
+        if (Ls == Lk) Dr = min(Ck0, d) - PbS;
     }
-    const int own2 = max(0, hibit(group_ballot<G>(first_sat, gbase)));
-    const int32_t Ck0 = PbS + (int32_t)(__shfl_sync(kFull, cinc, own2, G) & 0xffffu);
-    const int32_t Dr = ((Ls == Lk) ? min(Ck0, d) : d) - PbS;  // D - C at the row start
 
     // ---- level 2b: sub-blocks left of the one holding D count in full; that one in part
     const int ownD = hibit(group_ballot<G>(cb < Dr, gbase));  // -1 iff Dr <= 0 (then corr = 0)
