@@ -427,19 +427,23 @@ __global__ void __launch_bounds__(W * 32, 1) eval2_kernel(
                 lsum += v[i];
             }
             const uint32_t ex = group_incl_scan<G>(lsum, 0) - lsum;
-            uint32_t run = ex, cinc = 0;
-            const bool sat0 = ex <= key;
+            // C_{k0} matters only when the boundary row is k0's (Ls == Lk; else C_{k0} > d, D = d)
+            int32_t Dr = d - PbS;
+            if (__any_sync(kFull, Ls == Lk)) {
+                uint32_t run = ex, cinc = 0;
+                const bool sat0 = ex <= key;
 #pragma unroll
-            for (int i = 0; i < SPR; ++i) {
-                const bool sat = run <= key;
-                run += v[i];
-                cinc = sat ? run : cinc;
+                for (int i = 0; i < SPR; ++i) {
+                    const bool sat = run <= key;
+                    run += v[i];
+                    cinc = sat ? run : cinc;
+                }
+                const int own = max(0, hibit(group_ballot<G>(sat0, gbase)));
+                const int32_t Ck0 = PbS + (int32_t)(__shfl_sync(kFull, cinc, own, G) & 0xffffu);
+                if (Ls == Lk) Dr = min(Ck0, d) - PbS;
             }
-            const int own = max(0, hibit(group_ballot<G>(sat0, gbase)));
-            const int32_t Ck0 = PbS + (int32_t)(__shfl_sync(kFull, cinc, own, G) & 0xffffu);
-            const int32_t Dr = ((Ls == Lk) ? min(Ck0, d) : d) - PbS;
             int32_t corr = 0;
-            run = ex;
+            uint32_t run = ex;
 #pragma unroll
             for (int i = 0; i < SPR; ++i) {
                 const int32_t ci = (int32_t)(run & 0xffffu), si = (int32_t)(run >> 16);

@@ -377,18 +377,22 @@ __device__ __forceinline__ int32_t gchain_eval_cdd(const GChain<G, E>& ch, int l
         }
         const uint32_t ex = gscan<G>(lsum) - lsum;
         // k0: the last element of the row with S_excl <= Btot (a prefix of the row); its inclusive C
-        uint32_t run = ex, cinc = 0;
-        const bool sat0 = lane_in && ex <= key;
+        // (needed only when the boundary row is k0's, see boundary_two_level)
+        int32_t Dr = d - PbS;  // D - C at the row start
+        if (__any_sync(kFull, Ls == Lk)) {
+            uint32_t run = ex, cinc = 0;
+            const bool sat0 = lane_in && ex <= key;
 #pragma unroll
-        for (int i = 0; i < SPR; ++i) {
-            const bool sat = run <= key;
-            run += v[i];
-            cinc = sat ? run : cinc;
+            for (int i = 0; i < SPR; ++i) {
+                const bool sat = run <= key;
+                run += v[i];
+                cinc = sat ? run : cinc;
+            }
+            const int own = hibit(group_ballot<G>(sat0, gbase));  // >= 0: element 0 of the row has S = SbS
+            const int32_t Ck0 = PbS + (int32_t)(__shfl_sync(kFull, cinc, own < 0 ? 0 : own, G) & 0xffffu);
+            if (Ls == Lk) Dr = min(Ck0, d) - PbS;
         }
-        const int own = hibit(group_ballot<G>(sat0, gbase));  // >= 0: element 0 of the row has S = SbS
-        const int32_t Ck0 = PbS + (int32_t)(__shfl_sync(kFull, cinc, own < 0 ? 0 : own, G) & 0xffffu);
-        const int32_t Dr = ((Ls == Lk) ? min(Ck0, d) : d) - PbS;  // D - C at the row start
-        run = ex;
+        uint32_t run = ex;
 #pragma unroll
         for (int i = 0; i < SPR; ++i) {
             const int32_t ci = (int32_t)(run & 0xffffu), si = (int32_t)(run >> 16);
