@@ -191,3 +191,21 @@ def test_dpso_both_kernels(lib, monkeypatch, kernel, n, particles, iters, proble
                           oracle.dpso_params(problem=P, particles=particles, iters=iters, seed=77 + n), trace=True)
     assert np.array_equal(res["gbest_trace"].cpu().numpy()[:iters], ref["gbest_trace"])
     assert (pen, gid) == (ref["E_best"], ref["id"]) and np.array_equal(perm, ref["best"])
+
+
+def test_dpso_more_particles_than_slots(lib):
+    # more particles than resident slots (n = 300: ~8200 slots on a B200): every CTA runs several
+    # batches per iteration, so the single-GPU publish must map a key's particle to the CTA that
+    # holds it across batches (slot rows by parity), and the swarm-best trace must still match
+    import torch
+
+    inst = gen.cdd_instance(300, 6, 0.6)
+    ins = lib.Instance.from_gen(inst)
+    P, iters, seed = 9001, 4, 0x5107
+    res = lib.dpso_run(ins, P, iters, seed=seed, trace=True)
+    torch.cuda.synchronize()
+    pen, perm, gid = lib.best_get(ins)
+    ref = oracle.dpso_run(oracle.Problem.from_instance(inst),
+                          oracle.dpso_params(particles=P, iters=iters, seed=seed), trace=True)
+    assert np.array_equal(res["gbest_trace"].cpu().numpy()[:iters], ref["gbest_trace"])
+    assert (pen, gid) == (ref["E_best"], ref["id"]) and np.array_equal(perm, ref["best"])
