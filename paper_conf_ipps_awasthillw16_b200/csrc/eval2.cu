@@ -133,7 +133,7 @@ __global__ void __launch_bounds__(W * 32, 1) eval2_kernel(
     const uint8_t* __restrict__ tab_m, const uint8_t* __restrict__ tab_x,
     const uint16_t* __restrict__ tab_g, int n, int npow2,
     int kc_log2, int32_t d, const int16_t* __restrict__ perms, int64_t ld, int64_t batch,
-    int64_t* __restrict__ out, int* __restrict__ err) {
+    int64_t* __restrict__ out, int* __restrict__ err, bool quad) {
     using X = E2<G, E>;
     constexpr int CPW = X::CPW, CPS = X::CPS, SPR = X::SPR;
     extern __shared__ __align__(16) uint8_t smem[];
@@ -454,14 +454,28 @@ __global__ void __launch_bounds__(W * 32, 1) eval2_kernel(
             issue(rg + 2 * gstep, st);
             // ---- F(C_m'): early weights left of lane Ls, tardy weights from it on
             const bool amode = l < Ls;
-            const uint32_t psel = amode ? 0x4044u : 0x4144u;
-            const uint32_t wsum = amode ? 0x00010001u : 0x01000100u;
             uint32_t s = 0, acc = 0;
+            if (quad) {
+                // max(alpha, beta) <= 85: the weight bytes of four positions as one word (PRMT
+                // from two pair words), their byte-wise exclusive prefixes by one IMAD, dotted with
+                // the P quad by IDP.4A (as the SA kernels' quad pass)
+                const uint32_t xsel = amode ? 0x6420u : 0x7531u;
 #pragma unroll
-            for (int j = 0; j < E / 2; ++j) {
-                const uint32_t f2 = s * 0x10001u + __byte_perm(abp[j], 0u, psel);
-                acc = (j & 1) ? __dp2a_hi(f2, pw[j >> 1], acc) : __dp2a_lo(f2, pw[j >> 1], acc);
-                s = __dp4a(abp[j], wsum, s);
+                for (int q = 0; q < E / 4; ++q) {
+                    const uint32_t x = __byte_perm(abp[2 * q], abp[2 * q + 1], xsel);
+                    acc = __dp4a(x * 0x01010100u, pw[q], acc);
+                    acc += s * __dp4a(pw[q], 0x01010101u, 0u);
+                    s = __dp4a(x, 0x01010101u, s);
+                }
+            } else {
+                const uint32_t psel = amode ? 0x4044u : 0x4144u;
+                const uint32_t wsum = amode ? 0x00010001u : 0x01000100u;
+#pragma unroll
+                for (int j = 0; j < E / 2; ++j) {
+                    const uint32_t f2 = s * 0x10001u + __byte_perm(abp[j], 0u, psel);
+                    acc = (j & 1) ? __dp2a_hi(f2, pw[j >> 1], acc) : __dp2a_lo(f2, pw[j >> 1], acc);
+                    s = __dp4a(abp[j], wsum, s);
+                }
             }
             const int32_t base = amode ? Ab : (Btot - Bb);
             const int32_t contrib = base * (int32_t)tP + (amode ? (int32_t)acc : -(int32_t)acc) + corr;
@@ -498,7 +512,8 @@ cudaError_t launch2(const Instance& I, const int16_t* perms, int64_t ld, int64_t
     if (blocks > sms) blocks = sms;
     if (blocks < 1) blocks = 1;
     kern<<<(unsigned)blocks, W * 32, total, s>>>(I.tab_ab16, I.tab_p, I.tab_m, I.tab_x, I.tab_g, I.n,
-                                                 npow2, kc_log2, I.d_eff, perms, ld, batch, out, I.err);
+                                                 npow2, kc_log2, I.d_eff, perms, ld, batch, out, I.err,
+                                                 !UCD && I.ab85_ok && !getenv("CDD_EVAL2_NO_QUAD"));
     return cudaGetLastError();
 }
 

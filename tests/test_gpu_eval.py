@@ -236,10 +236,10 @@ def test_instance_argument_errors(lib):
 
 @pytest.mark.parametrize("n", [40, 300, 313])
 def test_cdd_weights_above_85(lib, n):
-    # alpha, beta in (85, 200]: the batched evaluator takes the 16-bit pair pass (the byte-quad pass
-    # needs max(alpha, beta) <= 85); one instance per side of the threshold, same sequences
-    for lo, hi in ((86, 200), (0, 85)):
-        inst = gen.ranged_instance(n, 23 + lo, (1, 4), (lo, hi), (lo, hi), 0.4)
+    # alpha, beta in (85, 100]: the batched evaluator takes the 16-bit pair pass (the byte-quad pass
+    # needs max(alpha, beta) <= 85); one instance per side of the threshold (both on the fast path)
+    for lo, hi in ((86, 100), (0, 85)):
+        inst = gen.ranged_instance(n, 23 + lo, (1, 3), (lo, hi), (lo, hi), 0.4)
         ins = lib.Instance.from_gen(inst)
         assert not ins.wide
         perms = gen.random_perms(500, n, n + lo)
