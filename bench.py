@@ -36,6 +36,14 @@ WORKLOAD = ("config5: CDD n=1000, h in {{0.2,0.4,0.6,0.8}} (instance seed 1), {c
 INT_OPS_PER_ELEM = 6  # 3 prefix adds + subtract + select + multiply-add per job
 
 
+_T_START = time.time()
+
+
+def _log(msg):
+    """Progress on stderr (stdout carries only the JSON line)."""
+    print(f"[bench {time.time() - _T_START:7.1f}s] {msg}", file=sys.stderr, flush=True)
+
+
 def _peaks():
     try:
         return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
@@ -122,7 +130,7 @@ def run_reference(args):
     import gen
     import oracle
 
-    threads = os.cpu_count() or 1
+    threads = len(os.sched_getaffinity(0)) or os.cpu_count() or 1
     chains_per_thread, steps = 1, 4000  # ~0.1-0.3 s of CPU work per bench step
     insts = [oracle.Problem.from_instance(gen.cdd_instance(N_JOBS, INSTANCE_SEED, h)) for h in HS]
     T0s = [oracle.t0(pr, oracle.CDD, RUN_SEED, 200) for pr in insts]
@@ -139,6 +147,7 @@ def run_reference(args):
             [x.join() for x in ts]
         return time.perf_counter() - t
 
+    _log("warmup")
     for _ in range(args.warmup):
         one_step()
     dts = [one_step() for _ in range(args.steps)]
@@ -175,7 +184,7 @@ def cpu_baseline_sample(seconds=12.0):
     import numpy as np
     import oracle
 
-    threads = os.cpu_count() or 1
+    threads = len(os.sched_getaffinity(0)) or os.cpu_count() or 1
     inst = gen.cdd_instance(N_JOBS, INSTANCE_SEED, 0.4)
     pr = oracle.Problem.from_instance(inst)
     T0 = oracle.t0(pr, oracle.CDD, RUN_SEED, 200)
@@ -199,18 +208,33 @@ def cpu_baseline_sample(seconds=12.0):
     [x.start() for x in ts]
     [x.join() for x in ts]
     dt = time.perf_counter() - t
-    # batched evaluation (the cdd_eval_batch leg's workload: random sequences at n=1000), ~3 s
-    rows = max(threads, int(3.0 / per_eval) * threads)
+    # batched evaluation (the cdd_eval_batch leg's workload: random sequences at n=1000): one
+    # bounded batch (generating the sequences is single-threaded numpy, so its size must not grow
+    # with the core count), evaluated on all threads repeatedly for ~3 s
+    rows = min(256 * threads, 16384)
     perms = gen.random_perms(rows, N_JOBS, 7, ld=N_JOBS)
+    bounds = np.linspace(0, rows, threads + 1).astype(np.int64)
+    cnt = [0] * threads
+
+    def ework(tid):
+        a, b = int(bounds[tid]), int(bounds[tid + 1])
+        t1 = time.perf_counter()
+        while b > a and time.perf_counter() - t1 < 3.0:
+            oracle.eval_batch(pr, perms[a:b])
+            cnt[tid] += b - a
+
+    ts = [threading.Thread(target=ework, args=(i,)) for i in range(threads)]
     t = time.perf_counter()
-    oracle.eval_batch_threaded(pr, perms, threads=threads)
-    ev_rate = rows / (time.perf_counter() - t)
+    [x.start() for x in ts]
+    [x.join() for x in ts]
+    ev_rate = sum(cnt) / (time.perf_counter() - t)
+    reps = sum(cnt) // rows
     return {"value": done[0] / dt, "unit": "evals/s", "cores": threads, "kind": "oracle",
             "cpu_model": _cpu_model(), "single_thread_evals_per_s": single,
             "eval_batch_evals_per_s": ev_rate,
             "sample": f"{threads} host threads x 1 SA chain x {steps} steps, CDD n=1000 h=0.4 "
                       f"(T0 from 200 samples, excluded); {dt:.1f} s; single thread {st_steps} steps; "
-                      f"batched evaluation of {rows} random sequences on {threads} threads"}
+                      f"batched evaluation of {rows} random sequences x {reps} passes on {threads} threads"}
 
 
 # ------------------------------------------------------------------------------ GPU arm
@@ -228,6 +252,9 @@ def main():
     ap.add_argument("--no-configs", action="store_true")
     ap.add_argument("--no-quality", action="store_true")
     args = ap.parse_args()
+    if os.environ.get("CDD_BENCH_WATCHDOG"):  # dump every thread's stack if a phase hangs
+        import faulthandler
+        faulthandler.dump_traceback_later(int(os.environ["CDD_BENCH_WATCHDOG"]), exit=True)
     if args.impl == "reference":
         return run_reference(args)
 
@@ -287,6 +314,7 @@ def main():
             out.append(ins)
         return out
 
+    _log("warmup")
     for _ in range(args.warmup):
         one_step()
     torch.cuda.synchronize()
@@ -376,20 +404,26 @@ def main():
                                    f"{sm_max:.0f} MHz max clock; instructions per evaluation from ncu "
                                    f"(profiles/sa_kernel_issue.json)")})
 
+    _log("timed region done")
     extra = {}
+    _log("eval_batch")
     if rank == 0 and not args.no_eval:
         extra["eval_batch"] = bench_eval(lib, gens[1], dev, stream, peaks)
+    _log("other configs")
     if rank == 0 and not args.no_configs:
         extra["other_configs"] = bench_configs(lib, dev, stream)
+    _log("quality table")
     if rank == 0 and not args.no_quality:
         extra["quality_table"] = bench_quality(lib, dev, stream)
     if world > 1 and not args.no_configs:
         dm = bench_dpso_multi_gpu(lib, cdist, dev, rank, world)
         if rank == 0:
             extra["dpso_multi_gpu"] = dm
+    _log("e2e")
     e2e = None
     if not args.no_e2e:
         e2e = bench_e2e(lib, gens, chains, steps, rank, world, dev, stream, max(1, args.steps // 2))
+    _log("cpu baseline")
     cpu = None
     if rank == 0 and not args.no_cpu_baseline:  # after the timed region (also at N > 1)
         cpu = cpu_baseline_sample()
@@ -490,6 +524,7 @@ def bench_configs(lib, dev, stream):
     import gen
 
     out = {}
+    _log("  config 1: CDD n=10")
     # config 1: CDD n=10, h=0.4, seed 1 -- all 10! sequences + one 10k-step chain
     g1 = gen.cdd_instance(10, 1, 0.4)
     i1 = lib.Instance.from_gen(g1, device=dev.index)
@@ -501,6 +536,7 @@ def bench_configs(lib, dev, stream):
     out["config1"] = {"exhaustive_evals_per_s": allp.shape[0] / t, "exhaustive_ms": 1000 * t,
                       "optimum": int(o1.min().item()), "sa_10k_chain_ms": 1000 * t_sa,
                       "sa_best": pen}
+    _log("  config 2: CDD n=100, h in")
     # config 2: CDD n=100, h in {0.2..0.8} (instance 1): 1M random sequences + 4096 chains x 5000
     p2 = gen.random_perms_device(1 << 20, 100, 2, device=dev)
     o2 = torch.empty(p2.shape[0], dtype=torch.int64, device=dev)
@@ -513,6 +549,7 @@ def bench_configs(lib, dev, stream):
         sa.append(4096 * 5001 / dt)
     out["config2"] = {"eval_batch_evals_per_s": sum(ev) / len(ev), "sa_evals_per_s": sum(sa) / len(sa),
                       "workload": "n=100, 4 h x instance 1; 2^20 random sequences; 4096 chains x 5000 steps"}
+    _log("  config 3: UCDDCP n=200 unrestricted")
     # config 3: UCDDCP n=200 unrestricted, 16384 chains x 5000 steps
     i3 = lib.Instance.from_gen(gen.ucddcp_instance(200, 1), device=dev.index)
     ws = lib.sa_run(i3, 16384, 5000, problem="ucddcp", seed=0x5EED0003)["workspace"]
@@ -520,6 +557,7 @@ def bench_configs(lib, dev, stream):
                                            workspace=ws))
     out["config3"] = {"sa_evals_per_s": 16384 * 5001 / dt, "ms": 1000 * dt,
                       "workload": "UCDDCP n=200 (d = sum p), 16384 chains x 5000 steps"}
+    _log("  config 4: CDD n=500, h=0.6: DPSO")
     # config 4: CDD n=500, h=0.6: DPSO 8192 particles vs SA at equal wall time (1 GPU)
     i4 = lib.Instance.from_gen(gen.cdd_instance(500, 1, 0.6), device=dev.index)
     iters = 200
@@ -534,6 +572,7 @@ def bench_configs(lib, dev, stream):
                       "dpso_best": dpso_best, "sa_steps_equal_time": sa_steps, "sa_best": sa_best,
                       "workload": "CDD n=500 h=0.6, DPSO 8192 particles x 200 iterations (w=c1=c2=0.5) vs "
                                   "8192 SA chains for the same wall time, 1 GPU"}
+    _log("  synchronous SA (P:181-188)")
     # synchronous SA on the config-5 instance h=0.4: 65536 chains, M=50 x 100 levels
     # (5000 moves per chain, like SA_5000) vs asynchronous SA with the same moves
     i5 = lib.Instance.from_gen(gen.cdd_instance(N_JOBS, INSTANCE_SEED, 0.4), device=dev.index)
@@ -546,6 +585,7 @@ def bench_configs(lib, dev, stream):
                       "async_best_same_moves": async_best,
                       "workload": "synchronous SA, CDD n=1000 h=0.4, 65536 chains, M=50 moves x 100 "
                                   "temperature levels (mu per level)"}
+    _log("  the headline SA from one V-shaped")
     # the headline SA from one V-shaped constructive sequence per chain instead of random ones
     # (sa_params.init; R13): quality only, same kernel and speed
     sys.path.insert(0, os.path.join(ROOT, "scripts"))
@@ -599,6 +639,7 @@ def bench_quality(lib, dev, stream):
 
     out = {}
     t0 = time.time()
+    _log("  config 2: CDD n=100, 10 instances")
     # config 2: CDD n=100, 10 instances x 4 h, 4096 chains x 5000 steps
     per_h = {f"{h:.1f}": [] for h in HS}
     for k in range(1, 11):
@@ -609,6 +650,7 @@ def bench_quality(lib, dev, stream):
             per_h[f"{h:.1f}"].append(gap(g, lib.best_get(ins)[0]))
     out["config2"] = summary(sum(per_h.values(), []), per_h={k: summary(v)["mean_gap_pct"] for k, v in per_h.items()},
                              workload="CDD n=100, 10 instances x 4 h, SA 4096 chains x 5000 steps")
+    _log("  config 3: UCDDCP n=200, 10 instances")
     # config 3: UCDDCP n=200, 10 instances, 16384 chains x 5000 steps
     rows = []
     for k in range(1, 11):
@@ -617,6 +659,7 @@ def bench_quality(lib, dev, stream):
         lib.sa_run(ins, 16384, 5000, problem="ucddcp", seed=0x5EED0003)
         rows.append(gap(g, lib.best_get(ins)[0]))
     out["config3"] = summary(rows, workload="UCDDCP n=200 (d = sum p), 10 instances, SA 16384 chains x 5000 steps")
+    _log("  config 4: CDD n=500 h=0.6, 10 instance")
     # config 4: CDD n=500 h=0.6, 10 instances: DPSO 8192 x 200 vs SA for the same wall time
     rd, rs = [], []
     for k in range(1, 11):
@@ -631,6 +674,7 @@ def bench_quality(lib, dev, stream):
     out["config4"] = {"dpso": summary(rd), "sa_equal_time": summary(rs),
                       "workload": "CDD n=500 h=0.6, 10 instances; DPSO 8192 particles x 200 iterations "
                                   "(w=c1=c2=0.5) vs 8192 SA chains for the same wall time"}
+    _log("  config 5: CDD n=1000, 10 instances")
     # config 5: CDD n=1000, 10 instances x 4 h, 65536 chains x 5000 steps (the headline workload)
     per_h = {f"{h:.1f}": [] for h in HS}
     for k in range(1, 11):
@@ -641,6 +685,7 @@ def bench_quality(lib, dev, stream):
             per_h[f"{h:.1f}"].append(gap(g, lib.best_get(ins)[0]))
     out["config5"] = summary(sum(per_h.values(), []), per_h={k: summary(v)["mean_gap_pct"] for k, v in per_h.items()},
                              workload=f"CDD n=1000, 10 instances x 4 h, SA {CHAINS} chains x {SA_STEPS} steps")
+    _log("  the other neighbourhoods")
     # the other neighbourhoods on the same 40 instances (R11b insertion, R11c contiguous window of
     # Pert = 4 positions; swap) beside the paper's Pert-FY reading R11 above
     moves = {}

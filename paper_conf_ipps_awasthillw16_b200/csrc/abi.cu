@@ -164,6 +164,7 @@ int cdd_instance_create(int32_t n, const int32_t* p, const int32_t* alpha, const
         return fail(CDD_EINVAL, "invalid CUDA device");
     int64_t sp = 0, sa = 0, sb = 0, sg = 0, sx = 0;
     int32_t pmax = 0, amax = 0, bmax = 0, mmax = 0, xmax = 0, gmax = 0;
+    int64_t smax = 0;  // max(alpha_i + beta_i)
     for (int i = 0; i < n; ++i) {
         if (p[i] < 1) return fail(CDD_EINVAL, "p_i must be >= 1");
         if (alpha[i] < 0 || beta[i] < 0) return fail(CDD_EINVAL, "alpha_i, beta_i must be >= 0");
@@ -173,6 +174,7 @@ int cdd_instance_create(int32_t n, const int32_t* p, const int32_t* alpha, const
         pmax = std::max(pmax, p[i]);
         amax = std::max(amax, alpha[i]);
         bmax = std::max(bmax, beta[i]);
+        smax = std::max(smax, (int64_t)alpha[i] + beta[i]);
         if (m) {
             if (m[i] < 0 || m[i] > p[i]) return fail(CDD_EINVAL, "need 0 <= m_i <= p_i");
             if (gamma[i] < 0) return fail(CDD_EINVAL, "gamma_i must be >= 0");
@@ -286,6 +288,7 @@ int cdd_instance_create(int32_t n, const int32_t* p, const int32_t* alpha, const
     chk(cudaMalloc(&I->tab_p, n));
     I->ab16_ok = amax <= 255 && bmax <= 255;
     I->ab85_ok = amax <= 85 && bmax <= 85;
+    I->s85_ok = I->ab85_ok && smax <= 85;
     std::vector<uint16_t> tab16(n);
     for (int i = 0; i < n; ++i) tab16[i] = (uint16_t)((alpha[i] & 0xff) | ((beta[i] & 0xff) << 8));
     chk(cudaMalloc(&I->tab_ab16, sizeof(uint16_t) * n));

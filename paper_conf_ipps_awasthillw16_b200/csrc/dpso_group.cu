@@ -54,7 +54,7 @@ struct DgArgs {
     unsigned long long* fkey;   // [2] = counter + 4: the single-GPU publish's running minima
     int64_t* trace;
     int np;
-    bool quad;  // CDD with max(alpha, beta) <= 85 (the evaluator's quad pass)
+    int quad;  // CDD: the evaluator's quad level (Instance::quad_level)
     // tables by job id (global; staged in shared memory per CTA): CDD alpha|beta<<8 | p<<16;
     // UCDDCP alpha|beta<<8 | gamma<<16 and M | X<<8
     const uint16_t* ab16;
@@ -441,7 +441,7 @@ __device__ __forceinline__ uint2 dg_build(const GChain<DG, E, UCD>& ch, const ui
 
 template <int DG, int E, bool UCD>
 __device__ __forceinline__ int32_t dg_eval(const GChain<DG, E, UCD>& ch, int l, int gbase, int n, int32_t d, uint2 t,
-                                          bool quad) {
+                                          int quad) {
     if constexpr (UCD)
         return gchain_eval_ucddcp<DG, E>(ch, l, gbase, n, t.x);
     else
@@ -893,7 +893,7 @@ static DgArgs dg_args(const Instance& I, const DpsoLaunch& p, const DpsoWsPtrs& 
     }
     a.trace = p.gbest_trace;
     a.np = w.np;
-    a.quad = I.ab85_ok && !getenv("CDD_SA_NO_QUAD");
+    a.quad = I.quad_level();
     a.ab16 = I.tab_ab16;
     a.p = I.tab_p;
     a.m = I.tab_m;

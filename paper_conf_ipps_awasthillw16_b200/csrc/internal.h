@@ -4,6 +4,7 @@
 
 #include <cstddef>
 #include <cstdint>
+#include <cstdlib>
 #include <vector>
 
 namespace cdd {
@@ -51,6 +52,13 @@ struct Instance {
     uint16_t* tab_ab16 = nullptr;  // alpha | beta << 8 (only when both <= 255: ab16_ok)
     bool ab16_ok = false;
     bool ab85_ok = false;  // max(alpha, beta) <= 85: the CDD evaluator's quad pass (sa_group.cuh)
+    bool s85_ok = false;   // also max(alpha + beta) <= 85: quad pass of the boundary row's level 1
+    // quad level of the group evaluators: 0 pairs, 1 quad pass, 2 also the quad boundary level 1
+    // (CDD_SA_NO_QUAD / CDD_SA_NO_QUAD2 cap it for experiments)
+    int quad_level() const {
+        if (!ab85_ok || std::getenv("CDD_SA_NO_QUAD")) return 0;
+        return (s85_ok && !std::getenv("CDD_SA_NO_QUAD2")) ? 2 : 1;
+    }
     uint32_t smem_base = 1024;  // shared-window address of dynamic shared memory (probed at create)
     uint8_t* tab_p = nullptr;
     uint8_t* tab_m = nullptr;

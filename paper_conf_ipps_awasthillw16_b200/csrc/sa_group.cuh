@@ -231,7 +231,7 @@ __device__ __forceinline__ void load_spread(const C& ch, int ls, int e0, bool in
 template <int G, int E>
 __device__ __forceinline__ int32_t boundary_two_level(const GChain<G, E>& ch, int l, int gbase,
                                                       int Ls, int Lk, int32_t d, int32_t PbS,
-                                                      int32_t thr, uint32_t key) {
+                                                      int32_t thr, uint32_t key, int quad) {
     using C = GChain<G, E>;
     constexpr int SB = E / G;   // positions per sub-block (16 for E = 128, G = 8)
     constexpr int L2 = SB / G;  // positions per lane in level 2
@@ -240,20 +240,40 @@ __device__ __forceinline__ int32_t boundary_two_level(const GChain<G, E>& ch, in
     const uint8_t* brow = ch.b8() + Ls * C::RS;
     const uint8_t* prow = ch.pb() + Ls * C::RS;
     // ---- level 1
-    uint32_t w[SB / 2], q[SB / 4];
-    ab_pairs<SB>(arow + SB * l, brow + SB * l, w);
+    uint32_t q[SB / 4];
     load_b8<SB>(prow + SB * l, q);
-    uint32_t Pb1 = 0, Sb1 = 0, sig2 = 0, dot = 0;
+    uint32_t Pb1 = 0, Sb1 = 0, dot = 0;
+    if (quad == 2) {
+        // max(alpha + beta) <= 85: the alpha and beta words add bytewise without carries, and the
+        // byte-wise exclusive prefixes of a quad (<= 3 * 85) fit a byte -- the main pass's quad
+        // form on x = alpha + beta (one IMAD + IDP.4A per quad, the cross term s * P_quad)
+        uint32_t a[SB / 4], b[SB / 4];
+        load_b8<SB>(arow + SB * l, a);
+        load_b8<SB>(brow + SB * l, b);
 #pragma unroll
-    for (int j = 0; j < SB / 4; ++j) Pb1 = __dp4a(q[j], 0x01010101u, Pb1);
+        for (int j = 0; j < SB / 4; ++j) {
+            const uint32_t x = a[j] + b[j];
+            const uint32_t pq = __dp4a(q[j], 0x01010101u, 0u);
+            dot = __dp4a(x * 0x01010100u, q[j], dot);
+            dot += Sb1 * pq;
+            Sb1 = __dp4a(x, 0x01010101u, Sb1);
+            Pb1 += pq;
+        }
+    } else {
+        uint32_t w[SB / 2];
+        ab_pairs<SB>(arow + SB * l, brow + SB * l, w);
+        uint32_t sig2 = 0;
 #pragma unroll
-    for (int j = 0; j < SB / 2; ++j) {
-        // positions 2j, 2j+1: f2 = (s, s + s_{2j}) in 16-bit halves, dotted with (p_{2j}, p_{2j+1})
-        const uint32_t f2 = __dp4a(w[j], 0x00000101u, 0u) * 0x10000u + sig2;
-        dot = (j & 1) ? __dp2a_hi(f2, q[j >> 1], dot) : __dp2a_lo(f2, q[j >> 1], dot);
-        const uint32_t pair = __dp4a(w[j], 0x01010101u, 0u);
-        sig2 += pair * 0x10001u;
-        Sb1 += pair;
+        for (int j = 0; j < SB / 4; ++j) Pb1 = __dp4a(q[j], 0x01010101u, Pb1);
+#pragma unroll
+        for (int j = 0; j < SB / 2; ++j) {
+            // positions 2j, 2j+1: f2 = (s, s + s_{2j}) in 16-bit halves, dotted with (p_{2j}, p_{2j+1})
+            const uint32_t f2 = __dp4a(w[j], 0x00000101u, 0u) * 0x10000u + sig2;
+            dot = (j & 1) ? __dp2a_hi(f2, q[j >> 1], dot) : __dp2a_lo(f2, q[j >> 1], dot);
+            const uint32_t pair = __dp4a(w[j], 0x01010101u, 0u);
+            sig2 += pair * 0x10001u;
+            Sb1 += pair;
+        }
     }
     const uint32_t lsum = Pb1 | (Sb1 << 16);
     const uint32_t ex = gscan<G>(lsum) - lsum;  // c_b | s_b << 16 at the sub-block start
@@ -282,13 +302,15 @@ __device__ __forceinline__ int32_t boundary_two_level(const GChain<G, E>& ch, in
         return gscan<G>(tot) - tot + __shfl_sync(kFull, ex, blk, G);  // row-relative start
     };
     uint32_t v[L2];
-    uint32_t run;
+    uint32_t run, run0 = 0;
     // D - C at the row start.  C_{k0} matters only when the boundary row is k0's (Ls == Lk); when
     // d's row comes first (Lt < Lk), C_{k0} > d and D = d -- the usual case for restrictive due
     // dates -- so a warp whose chains all have Ls < Lk skips the search for C_{k0}
     int32_t Dr = d - PbS;
-    if (__any_sync(kFull, Ls == Lk)) {
+    const bool s2a = __any_sync(kFull, Ls == Lk);
+    if (s2a) {
         run = spread(own, v);
+        run0 = run;
         uint32_t cinc = 0;
         const bool first_sat = run <= key;
 #pragma unroll
@@ -304,7 +326,9 @@ __device__ __forceinline__ int32_t boundary_two_level(const GChain<G, E>& ch, in
 
     // ---- level 2b: sub-blocks left of the one holding D count in full; that one in part
     const int ownD = hibit(group_ballot<G>(cb < Dr, gbase));  // -1 iff Dr <= 0 (then corr = 0)
-    run = spread(max(ownD, 0), v);
+    // D = C_{k0} (the unrestrictive case) lies in k0's sub-block: level 2a's spread is re-used
+    if (!s2a || !__all_sync(kFull, max(ownD, 0) == own)) run = spread(max(ownD, 0), v);
+    else run = run0;
     int32_t corr = (l < ownD) ? full : 0;
 #pragma unroll
     for (int i = 0; i < L2; ++i) {
@@ -320,7 +344,7 @@ __device__ __forceinline__ int32_t boundary_two_level(const GChain<G, E>& ch, in
 // quad: max(alpha, beta) <= 85 (the byte-wise prefix of three weights never carries).
 template <int G, int E>
 __device__ __forceinline__ int32_t gchain_eval_cdd(const GChain<G, E>& ch, int l, int gbase, int n,
-                                                   int32_t d, uint32_t tAB, uint32_t tP, bool quad) {
+                                                   int32_t d, uint32_t tAB, uint32_t tP, int quad) {
     using C = GChain<G, E>;
     constexpr int SPR = C::SPR;
     const uint32_t iP = gscan<G>(tP);
@@ -401,7 +425,7 @@ __device__ __forceinline__ int32_t gchain_eval_cdd(const GChain<G, E>& ch, int l
             run += v[i];
         }
     } else {
-        corr = boundary_two_level<G, E>(ch, l, gbase, Ls, Lk, d, PbS, thr, key);
+        corr = boundary_two_level<G, E>(ch, l, gbase, Ls, Lk, d, PbS, thr, key, quad);
     }
 
     // ---- F(C_{m'}) = sum_j p_j * (exclusive prefix of x within the lane row), x = alpha in early

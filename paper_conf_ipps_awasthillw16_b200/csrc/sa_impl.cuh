@@ -210,8 +210,8 @@ struct SaGArgs {
     // quad-major space; chains split between two warps hand their state over through `hand`
     int64_t share;
     uint8_t* hand;
-    // CDD: max(alpha, beta) <= 85, the evaluator's quad pass applies (sa_group.cuh)
-    bool quad;
+    // CDD: the evaluator's quad level (Instance::quad_level, sa_group.cuh)
+    int quad;
 };
 
 // State of one chain handed from the warp that ran its first steps to the warp finishing it.
@@ -336,7 +336,7 @@ __device__ void gchain_init(const GChain<G, E, UCD>& ch, int16_t* cur, int n, ui
 
 template <int G, int E, bool UCD>
 __device__ __forceinline__ int32_t gchain_eval(const GChain<G, E, UCD>& ch, int l, int gbase, int n,
-                                               int32_t d, uint2 t, bool quad) {
+                                               int32_t d, uint2 t, int quad) {
     if constexpr (UCD)
         return gchain_eval_ucddcp<G, E>(ch, l, gbase, n, t.x);
     else
@@ -881,7 +881,7 @@ __global__ void __launch_bounds__(kGThreads, sag_min_blocks<G, E, UCD>()) sa_gro
 // resident at once than with a warp per sample.  Same words (tag T0, id = sample) and the same
 // evaluator as the SA chains, so Z is bit-identical to t0_sample_kernel's.
 template <int G, int E, bool UCD>
-__global__ void __launch_bounds__(kGThreads) t0_group_kernel(ChainTables T, int n, int32_t d, bool quad, uint64_t seed,
+__global__ void __launch_bounds__(kGThreads) t0_group_kernel(ChainTables T, int n, int32_t d, int quad, uint64_t seed,
                                                             int64_t samples, int16_t* scratch, int64_t* Z) {
     using C = GChain<G, E, UCD>;
     constexpr int CPW = 32 / G;
@@ -968,7 +968,7 @@ cudaError_t t0_group_impl(const Instance& I, uint64_t seed, int64_t samples, dou
     uint8_t* base = static_cast<uint8_t*>(ws);
     int64_t* Z = reinterpret_cast<int64_t*>(base + w.z_off);
     int16_t* scratch = reinterpret_cast<int16_t*>(base + w.t0s_off);
-    t0_group_kernel<G, E, UCD><<<(unsigned)blocks, kGThreads, smem, s>>>(tables(I, UCD), I.n, I.d_eff, I.ab85_ok, seed,
+    t0_group_kernel<G, E, UCD><<<(unsigned)blocks, kGThreads, smem, s>>>(tables(I, UCD), I.n, I.d_eff, I.quad_level(), seed,
                                                                        samples, scratch, Z);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return e;
@@ -1041,7 +1041,7 @@ cudaError_t sag_impl(Instance& I, const SaLaunch& p, void* ws, cudaStream_t s) {
     cudaError_t e = cudaMemsetAsync(I.best_key, 0xff, sizeof(unsigned long long), s);
     if (e != cudaSuccess) return e;
     SaGArgs a{};
-    a.quad = I.ab85_ok && !getenv("CDD_SA_NO_QUAD");
+    a.quad = I.quad_level();
     a.T = tables(I, UCD);
     a.n = I.n;
     a.d = I.d_eff;
@@ -1243,7 +1243,7 @@ cudaError_t sag_sync_level(Instance& I, const SaLaunch& p, int64_t j, int64_t* l
         if (e != cudaSuccess) return e;
     }
     SaGArgs a{};
-    a.quad = I.ab85_ok && !getenv("CDD_SA_NO_QUAD");
+    a.quad = I.quad_level();
     a.T = tables(I, UCD);
     a.n = I.n;
     a.d = I.d_eff;

@@ -245,6 +245,10 @@ EDGE = [
     (700, dict(p=(1, 20), alpha=(1, 10), beta=(1, 15), h=0.0)),
     (1000, dict(p=(1, 20), alpha=(1, 10), beta=(1, 15), h=1.2)),
     (1000, dict(p=(1, 3), alpha=(40, 60), beta=(40, 60), h=0.45)),
+    # alpha + beta in [78, 85]: the quad form of the boundary row's level 1 at its byte limit
+    # (three prefix bytes of 85 = 255); the case above (alpha + beta up to 120) takes the pairs
+    (1000, dict(p=(1, 3), alpha=(40, 45), beta=(38, 40), h=0.5)),
+    (600, dict(p=(1, 3), alpha=(40, 45), beta=(38, 40), h=0.9)),
 ]
 
 
