@@ -11,7 +11,12 @@ out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-so
                      capture_output=True, text=True).stdout
 rows = list(csv.reader(io.StringIO(out)))
 hdr = rows[1]
-data = rows[2:]
+# the first kernel of the report only (a report of several launches repeats the header)
+data = []
+for r in rows[2:]:
+    if len(r) < len(hdr) or r == hdr:
+        break
+    data.append(r)
 isrc = hdr.index("Source")
 scols = [i for i, c in enumerate(hdr) if c.startswith("stall_") and "Not Issued" not in c]
 tot_by = {hdr[i]: 0 for i in scols}
