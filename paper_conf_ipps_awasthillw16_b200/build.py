@@ -12,7 +12,7 @@ OUT = os.path.join(HERE, "libcdd.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 SOURCES = ["abi.cu", "eval.cu", "eval2.cu", "sa.cu", "dpso.cu", "schedule.cu", "sag_cdd.cu",
            "sag_cdd_tr.cu", "sag_ucd.cu", "sag_ucd_tr.cu", "sag_cdd_ins.cu", "sag_cdd_ins_tr.cu",
-           "sag_ucd_ins.cu", "sag_ucd_ins_tr.cu", "wide.cu", "dpso_group.cu"]
+           "sag_ucd_ins.cu", "sag_ucd_ins_tr.cu", "sag_cdd_nib.cu", "sag_cdd_nib_tr.cu", "wide.cu", "dpso_group.cu"]
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
          "-Xcompiler", "-fPIC", "-Xcompiler", "-fvisibility=hidden", "--expt-relaxed-constexpr",
          "-Xptxas", "-v"]

@@ -289,6 +289,7 @@ int cdd_instance_create(int32_t n, const int32_t* p, const int32_t* alpha, const
     I->ab16_ok = amax <= 255 && bmax <= 255;
     I->ab85_ok = amax <= 85 && bmax <= 85;
     I->s85_ok = I->ab85_ok && smax <= 85;
+    I->nib_ok = amax <= 15 && bmax <= 15 && (int64_t)pmax * std::max(amax, bmax) * 120 < 65536;
     std::vector<uint16_t> tab16(n);
     for (int i = 0; i < n; ++i) tab16[i] = (uint16_t)((alpha[i] & 0xff) | ((beta[i] & 0xff) << 8));
     chk(cudaMalloc(&I->tab_ab16, sizeof(uint16_t) * n));

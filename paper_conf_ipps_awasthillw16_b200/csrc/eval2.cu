@@ -267,7 +267,7 @@ __global__ void __launch_bounds__(W * 32, 1) eval2_kernel(
         }
         if constexpr (UCD) {
             // ---- gather: 16-bit alpha|beta<<8 pairs, gamma pairs, M and X bytes, lane totals
-            uint32_t abp[E / 2], gp[E / 2], mw[E / 4], xw[E / 4];
+            uint32_t abp[E / 2], gp[E / 2], mx[E / 2];
             uint32_t tA = 0, tB = 0;
 #pragma unroll
             for (int c = 0; c < CPS; ++c) {
@@ -289,13 +289,8 @@ __global__ void __launch_bounds__(W * 32, 1) eval2_kernel(
                     tB = __dp4a(a, 0x01000100u, tB);
                 }
 #pragma unroll
-                for (int h = 0; h < 2; ++h) {
-                    // (M0, M1, X0, X1), (M2, M3, X2, X3) -> M quad, X quad
-                    const uint32_t mx01 = __byte_perm(r[4 * h].y, r[4 * h + 1].y, 0x5140u);
-                    const uint32_t mx23 = __byte_perm(r[4 * h + 2].y, r[4 * h + 3].y, 0x5140u);
-                    mw[2 * c + h] = __byte_perm(mx01, mx23, 0x5410u);
-                    xw[2 * c + h] = __byte_perm(mx01, mx23, 0x7632u);
-                }
+                for (int j = 0; j < 4; ++j)  // (M_{2j}, M_{2j+1}, X_{2j}, X_{2j+1}): the pass's two IDP.2A
+                    mx[4 * c + j] = __byte_perm(r[2 * j].y, r[2 * j + 1].y, 0x5140u);
             }
             // ---- scan, boundary lane Lk (d >= sum P: the due date sits at C_{k0}; as gchain_eval_ucddcp)
             const uint32_t tAB = tA | (tB << 16);
@@ -352,13 +347,8 @@ __global__ void __launch_bounds__(W * 32, 1) eval2_kernel(
                 const uint32_t f2 = s * 0x10001u + __byte_perm(abp[j], 0u, psel);
                 const uint32_t w2 = f2 * sgn + base2;
                 const uint32_t mn2 = __vminu2(w2, gp[j]);
-                if (j & 1) {
-                    acc = __dp2a_hi(w2, mw[j >> 1], acc);
-                    acc = __dp2a_hi(mn2, xw[j >> 1], acc);
-                } else {
-                    acc = __dp2a_lo(w2, mw[j >> 1], acc);
-                    acc = __dp2a_lo(mn2, xw[j >> 1], acc);
-                }
+                acc = __dp2a_lo(w2, mx[j], acc);
+                acc = __dp2a_hi(mn2, mx[j], acc);
                 s = __dp4a(abp[j], wsum, s);
             }
             const int32_t Z = (int32_t)gsum2<G>(acc + (uint32_t)corr);

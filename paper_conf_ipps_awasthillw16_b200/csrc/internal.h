@@ -53,6 +53,9 @@ struct Instance {
     bool ab16_ok = false;
     bool ab85_ok = false;  // max(alpha, beta) <= 85: the CDD evaluator's quad pass (sa_group.cuh)
     bool s85_ok = false;   // also max(alpha + beta) <= 85: quad pass of the boundary row's level 1
+    // alpha, beta <= 15 and pmax * max(alpha, beta) * 120 < 2^16: the SA nibble layout with
+    // sub-block summaries (sa_nib.cuh) for n in (512, 1024]
+    bool nib_ok = false;
     // quad level of the group evaluators: 0 pairs, 1 quad pass, 2 also the quad boundary level 1
     // (CDD_SA_NO_QUAD / CDD_SA_NO_QUAD2 cap it for experiments)
     int quad_level() const {
@@ -196,6 +199,8 @@ struct GroupCfg {
                           unsigned long long** key, int16_t** perm);
 CDD_SAG_DECL(sag_cdd)
 CDD_SAG_DECL(sag_cdd_tr)
+CDD_SAG_DECL(sag_cdd_nib)
+CDD_SAG_DECL(sag_cdd_nib_tr)
 CDD_SAG_DECL(sag_ucd)
 CDD_SAG_DECL(sag_ucd_tr)
 CDD_SAG_DECL(sag_cdd_ins)

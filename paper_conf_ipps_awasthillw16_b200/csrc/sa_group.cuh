@@ -27,6 +27,10 @@
 #ifndef CDD_SAG_PREFETCH
 #define CDD_SAG_PREFETCH 0
 #endif
+// timing experiment only (wrong results): the CDD quad pass streams 1/CDD_SAG_PASSDIV of each row
+#ifndef CDD_SAG_PASSDIV
+#define CDD_SAG_PASSDIV 1
+#endif
 // 1: the CDD pass runs the two halves of a lane row as independent dependency chains (experiment)
 #ifndef CDD_SAG_SPLITPASS
 #define CDD_SAG_SPLITPASS 0
@@ -228,21 +232,19 @@ __device__ __forceinline__ void load_spread(const C& ch, int ls, int e0, bool in
 //  level 2: the sub-block holding k0 (last start with S <= Btot) is spread over the G lanes
 //           (SB/G positions each) to find C_{k0}, hence D; then the sub-block holding D (last start
 //           with c < D) is spread the same way for its partial term.
+// Level 1 of the byte-row layout: sub-block l of row Ls streamed (the nibble layout of sa_nib.cuh
+// reads a cached summary instead).
 template <int G, int E>
-__device__ __forceinline__ int32_t boundary_two_level(const GChain<G, E>& ch, int l, int gbase,
-                                                      int Ls, int Lk, int32_t d, int32_t PbS,
-                                                      int32_t thr, uint32_t key, int quad) {
+__device__ __forceinline__ void bt_level1(const GChain<G, E>& ch, int Ls, int l, int quad, uint32_t& Pb1,
+                                          uint32_t& Sb1, uint32_t& dot) {
     using C = GChain<G, E>;
-    constexpr int SB = E / G;   // positions per sub-block (16 for E = 128, G = 8)
-    constexpr int L2 = SB / G;  // positions per lane in level 2
-    static_assert(SB % 8 == 0 && L2 >= 1 && L2 <= 4, "two-level boundary layout");
+    constexpr int SB = E / G;
     const uint8_t* arow = ch.a8() + Ls * C::RS;
     const uint8_t* brow = ch.b8() + Ls * C::RS;
     const uint8_t* prow = ch.pb() + Ls * C::RS;
-    // ---- level 1
     uint32_t q[SB / 4];
     load_b8<SB>(prow + SB * l, q);
-    uint32_t Pb1 = 0, Sb1 = 0, dot = 0;
+    Pb1 = 0, Sb1 = 0, dot = 0;
     if (quad == 2) {
         // max(alpha + beta) <= 85: the alpha and beta words add bytewise without carries, and the
         // byte-wise exclusive prefixes of a quad (<= 3 * 85) fit a byte -- the main pass's quad
@@ -275,6 +277,48 @@ __device__ __forceinline__ int32_t boundary_two_level(const GChain<G, E>& ch, in
             Sb1 += pair;
         }
     }
+}
+
+// Level 2 of the byte-row layout: L2 consecutive positions from e (row-relative) of row Ls as
+// alpha|beta<<8 pair words and a P word.
+template <int L2, int G, int E>
+__device__ __forceinline__ void bt_spread_load(const GChain<G, E>& ch, int Ls, int e, uint32_t (&a2)[(L2 + 1) / 2],
+                                               uint32_t& pp) {
+    using C = GChain<G, E>;
+    const uint8_t* arow = ch.a8() + Ls * C::RS;
+    const uint8_t* brow = ch.b8() + Ls * C::RS;
+    const uint8_t* prow = ch.pb() + Ls * C::RS;
+    if constexpr (L2 >= 2) {
+        ab_pairs<L2>(arow + e, brow + e, a2);
+        pp = L2 == 4 ? *reinterpret_cast<const uint32_t*>(prow + e) : (uint32_t)*reinterpret_cast<const uint16_t*>(prow + e);
+    } else {
+        a2[0] = (uint32_t)arow[e] | ((uint32_t)brow[e] << 8);
+        pp = prow[e];
+    }
+}
+
+// Boundary row Ls for rows of E >= G^2 positions, in two levels, returning this lane's share of
+// corr = sum_k (S_k - Btot) * clamp(D - C_{k-1}, 0, p_k) over the row (row-relative: c_k, s_k
+// exclusive prefixes of p and alpha + beta, thr = Btot - S at the row start).
+//  level 1: lane l takes sub-block l (SB = E/G consecutive positions): its sums of p and
+//           alpha + beta (IDP.4A), its local dot  sum_k p_k * s^loc_k  (f2 pairs + IDP.2A), and a
+//           G-lane scan of the packed sums gives every sub-block's start.  Sub-blocks wholly left
+//           of D contribute  dot + (s_b - thr) * P_b  each.
+//  level 2: the sub-block holding k0 (last start with S <= Btot) is spread over the G lanes
+//           (SB/G positions each) to find C_{k0}, hence D; then the sub-block holding D (last start
+//           with c < D) is spread the same way for its partial term.
+// The layout's loads are the bt_level1 / bt_spread_load overloads (GChain here, GChainNib in
+// sa_nib.cuh).
+template <int G, int E, class C>
+__device__ __forceinline__ int32_t boundary_two_level(const C& ch, int l, int gbase,
+                                                      int Ls, int Lk, int32_t d, int32_t PbS,
+                                                      int32_t thr, uint32_t key, int quad) {
+    constexpr int SB = E / G;   // positions per sub-block (16 for E = 128, G = 8)
+    constexpr int L2 = SB / G;  // positions per lane in level 2
+    static_assert(SB % 8 == 0 && L2 >= 1 && L2 <= 4, "two-level boundary layout");
+    // ---- level 1
+    uint32_t Pb1, Sb1, dot;
+    bt_level1(ch, Ls, l, quad, Pb1, Sb1, dot);
     const uint32_t lsum = Pb1 | (Sb1 << 16);
     const uint32_t ex = gscan<G>(lsum) - lsum;  // c_b | s_b << 16 at the sub-block start
     const int32_t cb = (int32_t)(ex & 0xffffu), sb = (int32_t)(ex >> 16);
@@ -285,13 +329,7 @@ __device__ __forceinline__ int32_t boundary_two_level(const GChain<G, E>& ch, in
     auto spread = [&](int blk, uint32_t (&v)[L2]) -> uint32_t {
         const int e = SB * blk + L2 * l;
         uint32_t a2[(L2 + 1) / 2], pp;
-        if constexpr (L2 >= 2) {
-            ab_pairs<L2>(arow + e, brow + e, a2);
-            pp = L2 == 4 ? *reinterpret_cast<const uint32_t*>(prow + e) : (uint32_t)*reinterpret_cast<const uint16_t*>(prow + e);
-        } else {
-            a2[0] = (uint32_t)arow[e] | ((uint32_t)brow[e] << 8);
-            pp = prow[e];
-        }
+        bt_spread_load<L2>(ch, Ls, e, a2, pp);
         uint32_t tot = 0;
 #pragma unroll
         for (int i = 0; i < L2; ++i) {
@@ -439,7 +477,7 @@ __device__ __forceinline__ int32_t gchain_eval_cdd(const GChain<G, E>& ch, int l
         // per quad: byte-wise exclusive prefixes [0, x0, x0+x1, x0+x1+x2] by one IMAD, their dot
         // with the P quad by IDP.4A, plus s * (sum of the P quad)
 #pragma unroll
-        for (int c0 = 0; c0 < E; c0 += CH) {
+        for (int c0 = 0; c0 < E / CDD_SAG_PASSDIV; c0 += CH) {
             uint32_t x[CH / 4], q[CH / 4];
             load_b8<CH>(xrow + c0, x);
             load_b8<CH>(prow + c0, q);

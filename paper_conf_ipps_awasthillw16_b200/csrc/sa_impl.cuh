@@ -14,6 +14,7 @@
 #include "internal.h"
 #include "peer.cuh"
 #include "sa_group.cuh"
+#include "sa_nib.cuh"
 
 namespace cdd {
 namespace {
@@ -167,9 +168,22 @@ __global__ void t0_reduce_kernel(const int64_t* __restrict__ Z, int64_t N, doubl
 #endif
 // resident CTAs the register budget is sized for: as many as shared memory admits, at most
 // CDD_SAG_MIN_BLOCKS (UCDDCP at E = 64 holds 58 KB of chains per CTA -> 3)
-template <int G, int E, bool UCD>
+// the chain layout of a group-kernel variant: MV = 2 is the nibble layout with sub-block
+// summaries (sa_nib.cuh; CDD, moves of <= 4 positions, G = 8, E = 128)
+template <int G, int E, bool UCD, int MV>
+struct SagChainT {
+    using type = GChain<G, E, UCD>;
+};
+template <int G, int E>
+struct SagChainT<G, E, false, 2> {
+    using type = GChainNib<G, E>;
+};
+template <int G, int E, bool UCD, int MV>
+using SagChain = typename SagChainT<G, E, UCD, MV>::type;
+
+template <int G, int E, bool UCD, int MV = 0>
 constexpr int sag_min_blocks() {
-    constexpr int per_cta = 4 * (32 / G) * GChain<G, E, UCD>::BYTES + 2048;
+    constexpr int per_cta = 4 * (32 / G) * SagChain<G, E, UCD, MV>::BYTES + 2048;
     constexpr int fit = (228 * 1024) / per_cta;
     return fit < 1 ? 1 : (fit < CDD_SAG_MIN_BLOCKS ? fit : CDD_SAG_MIN_BLOCKS);
 }
@@ -252,14 +266,12 @@ __device__ __forceinline__ uint2 gchain_lane_totals(const GChain<G, E, UCD>& ch,
     return make_uint2(tAB, tP);
 }
 
-template <int G, int E, bool UCD>
-__device__ void gchain_init(const GChain<G, E, UCD>& ch, int16_t* cur, int n, uint64_t seed,
-                            uint64_t g, int l, const ChainTables& T, const int16_t* init, int* err,
-                            uint32_t tag = kTagSaInit) {
-    using C = GChain<G, E, UCD>;
-    constexpr int NP = C::NP;
-    // staging: NP ids then 4G Philox words, 2 NP + 16 G bytes <= C::BYTES (static_assert there)
-    uint16_t* ids = reinterpret_cast<uint16_t*>(ch.base);
+// Alg. 1 line 1, the sequence: Fisher-Yates of the identity (or the caller's sequence) staged in
+// the chain's shared memory at base (NP ids then 4G Philox words), copied to the global slot cur.
+template <int G, int NP>
+__device__ void gchain_ids(uint8_t* base, int16_t* cur, int n, uint64_t seed, uint64_t g, int l,
+                           const int16_t* init, int* err, uint32_t tag) {
+    uint16_t* ids = reinterpret_cast<uint16_t*>(base);
     uint32_t* words = reinterpret_cast<uint32_t*>(ids + NP);
     if (init)
         for (int k = l; k < NP; k += G) {
@@ -307,6 +319,16 @@ __device__ void gchain_init(const GChain<G, E, UCD>& ch, int16_t* cur, int n, ui
     __syncwarp();
     for (int k = l; k < NP; k += G) cur[k] = (int16_t)ids[k];
     __syncwarp();
+}
+
+template <int G, int E, bool UCD>
+__device__ void gchain_init(const GChain<G, E, UCD>& ch, int16_t* cur, int n, uint64_t seed,
+                            uint64_t g, int l, const ChainTables& T, const int16_t* init, int* err,
+                            uint32_t tag = kTagSaInit) {
+    using C = GChain<G, E, UCD>;
+    constexpr int NP = C::NP;
+    // staging: NP ids then 4G Philox words, 2 NP + 16 G bytes <= C::BYTES (static_assert there)
+    gchain_ids<G, NP>(ch.base, cur, n, seed, g, l, init, err, tag);
     // records in batches of 8 positions per lane: 8 independent id loads, then 8 independent
     // table loads (E is a multiple of 8, so NP is a multiple of 8 G)
     for (int k0 = l; k0 < NP; k0 += 8 * G) {
@@ -332,6 +354,58 @@ __device__ void gchain_init(const GChain<G, E, UCD>& ch, int16_t* cur, int n, ui
     __syncwarp();
     ch.tot()[l] = gchain_lane_totals(ch, l);
     __syncwarp();
+}
+
+// The nibble layout (sa_nib.cuh): records alpha | beta << 4 and P, lane totals, and the summaries
+// of the lane's 8 sub-blocks.
+template <int G, int E, bool UCD>
+__device__ void gchain_init(const GChainNib<G, E>& ch, int16_t* cur, int n, uint64_t seed,
+                            uint64_t g, int l, const ChainTables& T, const int16_t* init, int* err,
+                            uint32_t tag = kTagSaInit) {
+    using C = GChainNib<G, E>;
+    constexpr int NP = C::NP;
+    gchain_ids<G, NP>(ch.base, cur, n, seed, g, l, init, err, tag);
+    for (int k0 = l; k0 < NP; k0 += 8 * G) {
+        int jj[8];
+#pragma unroll
+        for (int u = 0; u < 8; ++u) jj[u] = k0 + u * G < n ? cur[k0 + u * G] : 0;
+#pragma unroll
+        for (int u = 0; u < 8; ++u) {
+            const int k = k0 + u * G;
+            const bool v = k < n;
+            const uint32_t ab = v ? __ldg(T.ab16 + jj[u]) : 0u;
+            ch.ab()[k] = (uint8_t)((ab & 15u) | ((ab >> 4) & 0xf0u));
+            ch.pb()[k] = v ? __ldg(T.p + jj[u]) : (uint8_t)0;
+        }
+    }
+    __syncwarp();
+    uint32_t tA = 0, tB = 0, tP = 0;
+#pragma unroll
+    for (int b = 0; b < C::NSB; ++b) {
+        const uint2 sm = nib_summary(ch, l * E + 16 * b);
+        ch.sum()[b * G + l] = sm;
+        tA += sm.y & 0xffu;
+        tB += (sm.y >> 8) & 0xffu;
+        tP += sm.y >> 16;
+    }
+    ch.tot()[l] = make_uint2(tA | (tB << 16), tP);
+    __syncwarp();
+}
+
+template <int G, int E, bool UCD>
+__device__ __forceinline__ int32_t gchain_eval(const GChainNib<G, E>& ch, int l, int gbase, int n,
+                                               int32_t d, uint2 t, int quad) {
+    return gchain_eval_nib<G, E>(ch, l, gbase, n, d, t.x, t.y, quad);
+}
+
+template <int G, int E, bool UCD>
+__device__ __forceinline__ uint2 pos_read(const GChainNib<G, E>& ch, int k) {
+    return make_uint2(nib_read(ch, k), 0u);
+}
+
+template <int G, int E, bool UCD>
+__device__ __forceinline__ void pos_write(const GChainNib<G, E>& ch, int k, uint2 v) {
+    nib_write(ch, k, v.x);
 }
 
 template <int G, int E, bool UCD>
@@ -606,10 +680,11 @@ __device__ __forceinline__ uint2 rot_tot_delta(const GChain<G, E, UCD>& ch, int 
     return make_uint2(ab_wide(i.x & 0xffffu) - ab_wide(o.x & 0xffffu), pi - po);
 }
 
-// MV: 0 = moves of <= 4 positions (Pert-FY, swap, window), 1 = insertion (a segment rotation)
+// MV: 0 = moves of <= 4 positions (Pert-FY, swap, window), 1 = insertion (a segment rotation),
+// 2 = moves of <= 4 positions on the nibble layout with sub-block summaries (sa_nib.cuh)
 template <int G, int E, bool UCD, bool TRACE, int MV>
-__global__ void __launch_bounds__(kGThreads, sag_min_blocks<G, E, UCD>()) sa_group_kernel(SaGArgs a) {
-    using C = GChain<G, E, UCD>;
+__global__ void __launch_bounds__(kGThreads, sag_min_blocks<G, E, UCD, MV>()) sa_group_kernel(SaGArgs a) {
+    using C = SagChain<G, E, UCD, MV>;
     constexpr int NP = C::NP;
     constexpr int CPW = 32 / G;   // chains per warp
     constexpr int SPG = G / 2;    // steps of moves per precompute
@@ -750,6 +825,14 @@ __global__ void __launch_bounds__(kGThreads, sag_min_blocks<G, E, UCD>()) sa_gro
             const bool mover = l < P;
             const int myq = mover ? (int)(((l < 2 ? q01 : q23) >> (16 * (l & 1))) & 0xffffu) : 0;
             const uint2 old_v = pos_read<G, E, UCD>(ch, myq);
+            // nibble layout: the summary of the mover's sub-block (every mover reads before any
+            // writes; movers sharing a sub-block write the same values)
+            uint2 old_s = make_uint2(0u, 0u);
+            int sidx = 0;
+            if constexpr (MV == 2) {
+                sidx = C::sidx(myq);
+                old_s = ch.sum()[sidx];
+            }
             // unconditional (myq = 0 for non-movers): consumed only after the evaluation
             const int16_t old_id = cur[myq];
             const int src = (int)((sig >> (2 * (l & 3))) & 3u);
@@ -764,6 +847,10 @@ __global__ void __launch_bounds__(kGThreads, sag_min_blocks<G, E, UCD>()) sa_gro
                 if constexpr (!UCD) atomicAdd(t2 + 1, (new_v.x >> 16) - (old_v.x >> 16));
             }
             __syncwarp();
+            if constexpr (MV == 2) {
+                if (mover) ch.sum()[sidx] = nib_summary(ch, myq & ~15);
+                __syncwarp();
+            }
             const uint2 tn = ch.tot()[l];
             // line 6
             const int32_t En = gchain_eval<G, E, UCD>(ch, l, gbase, n, a.d, tn, a.quad);
@@ -794,7 +881,10 @@ __global__ void __launch_bounds__(kGThreads, sag_min_blocks<G, E, UCD>()) sa_gro
                 }
                 Ecur = En;
             } else {
-                if (mover) pos_write<G, E, UCD>(ch, myq, old_v);
+                if (mover) {
+                    pos_write<G, E, UCD>(ch, myq, old_v);
+                    if constexpr (MV == 2) ch.sum()[sidx] = old_s;
+                }
                 ch.tot()[l] = tt;
             }
             __syncwarp();
@@ -980,7 +1070,7 @@ cudaError_t t0_group_impl(const Instance& I, uint64_t seed, int64_t samples, dou
 template <int G, int E, bool UCD, bool TRACE, int MV>
 Grid sag_grid(const Instance& I, int64_t chains) {
     constexpr int CPB = kGWarps * (32 / G);  // chains per CTA
-    Grid gr{1, (size_t)CPB * GChain<G, E, UCD>::BYTES};
+    Grid gr{1, (size_t)CPB * SagChain<G, E, UCD, MV>::BYTES};
     int sms = 148, occ = 1;
     resident_ctas(reinterpret_cast<const void*>(sa_group_kernel<G, E, UCD, TRACE, MV>), I.device, kGThreads, gr.smem,
                   &sms, &occ);
@@ -1345,6 +1435,16 @@ int pow2_at_least(int c) {
         uint8_t* base = static_cast<uint8_t*>(ws);                                               \
         *key = reinterpret_cast<unsigned long long*>(base + w.keys_off) + 1;                     \
         *perm = reinterpret_cast<int16_t*>(base + w.smin_off);                                   \
+    }
+
+// The nibble-layout variant (MV = 2, sa_nib.cuh): CDD, G = 8, E = 128 only.
+#define CDD_SAG_NIB_VARIANT(NAME, TR)                                                             \
+    size_t NAME##_ws(const Instance& I, const SaLaunch& p, GroupCfg cfg) {                       \
+        return cfg.G == 8 && cfg.E == 128 ? sag_ws<8, 128, false, TR, 2>(I, p) : 0;              \
+    }                                                                                            \
+    cudaError_t NAME##_run(Instance& I, const SaLaunch& p, GroupCfg cfg, void* ws, cudaStream_t s) { \
+        return cfg.G == 8 && cfg.E == 128 ? sag_impl<8, 128, false, TR, 2>(I, p, ws, s)           \
+                                          : cudaErrorInvalidValue;                               \
     }
 
 #define CDD_SAG_T0_VARIANT(NAME, UCD)                                                             \

@@ -430,3 +430,58 @@ def test_balanced_schedule_every_chain(lib, problem, n, chains, steps):
         assert np.array_equal(r2["chain_best"].cpu().numpy(), cb)
     finally:
         del os.environ["CDD_SA_BALANCE"]
+
+
+# The nibble layout with sub-block summaries (csrc/sa_nib.cuh): CDD with alpha, beta <= 15 and
+# pmax * max(alpha, beta) * 120 < 2^16 at G = 8, E = 128 (n in (512, 1024]).  Every move of <= 4
+# positions, traced chain by chain against the oracle, and the same run with the byte-row layout
+# (CDD_SA_NO_NIB=1) must give the identical trace.  The instances put the 16-bit sub-block forms
+# at their limit (p up to 36 with weights 15: 36 * 15 * 120 = 64800) and n off the sub-block grid.
+NIB = [
+    (1000, dict(p=(1, 20), alpha=(1, 10), beta=(1, 15), h=0.4)),
+    (777, dict(p=(30, 36), alpha=(14, 15), beta=(13, 15), h=0.6)),
+    (530, dict(p=(1, 36), alpha=(0, 15), beta=(0, 15), h=0.2)),
+]
+
+
+@pytest.mark.parametrize("n,kw", NIB)
+@pytest.mark.parametrize("move,pert", [("pert_fy", 4), ("pert_fy", 3), ("swap", 2), ("window", 4)])
+def test_nibble_layout_trace_parity(lib, n, kw, move, pert):
+    inst = gen.ranged_instance(n, 5, **kw)
+    chains, steps, seed = 48, 150, 77 + n
+    ins, res, (pen, perm, gid), pr, p, T0 = _run_both(lib, inst, "cdd", chains, steps, seed, samples=300,
+                                                     move=move, pert=pert, lanes=8)
+    assert lib.sa_layout(ins, chains, lanes=8) == (8, 128)
+    tr = res["trace"].cpu().numpy()
+    for c in range(chains):
+        ref = oracle.sa_chain(pr, p, T0, c, trace=True)
+        assert np.array_equal(tr[c] >> 1, ref["E_new"]), c
+        assert np.array_equal((tr[c] & 1).astype(bool), ref["accepted"]), c
+    full = oracle.sa_run(pr, p, T0)
+    assert (pen, gid) == (full["E_best"], full["g"]) and np.array_equal(perm, full["best"])
+    os.environ["CDD_SA_NO_NIB"] = "1"
+    try:
+        res2 = lib.sa_run(lib.Instance.from_gen(inst), chains, steps, T0=T0, pert=pert, move=move,
+                          seed=seed, trace=True, lanes=8)
+    finally:
+        del os.environ["CDD_SA_NO_NIB"]
+    assert np.array_equal(res2["trace"].cpu().numpy(), tr)
+
+
+def test_nibble_layout_full_grid_and_balanced(lib):
+    # many chains (G = 8 by the automatic layout): every chain's best and final penalty against
+    # the oracle, round robin over more chains than resident slots and the balanced schedule
+    import torch
+
+    inst = gen.cdd_instance(1000, 3, 0.6)
+    pr = _prob(inst)
+    for chains in (70000, 73040):
+        ins = lib.Instance.from_gen(inst)
+        res = lib.sa_run(ins, chains, 40, T0=500.0, seed=11, chain_best=True, chain_final=True)
+        torch.cuda.synchronize()
+        assert lib.sa_layout(ins, chains) == (8, 128)
+        cb, cf = res["chain_best"].cpu().numpy(), res["chain_final"].cpu().numpy()
+        p = oracle.sa_params(chains=1, steps=40, seed=11)
+        for c in list(range(0, chains, 997)) + [chains - 1]:
+            ref = oracle.sa_chain(pr, p, 500.0, c)
+            assert (cb[c], cf[c]) == (ref["E_best"], ref["E_final"]), c
