@@ -374,7 +374,9 @@ def main():
         traffic = json.load(open(tp)).get("dram_bytes_per_launch")
     step_ms = ms / args.steps
     G, E = lib.sa_layout(insts[0], chains)
-    kname = (f"sa_group_kernel<{G},{E}> (CDD, {32 // G} chains per warp)" if G < 32
+    nib = (G, E) == (8, 128) and insts[0].query()["small_weights"] and not os.environ.get("CDD_SA_NO_NIB")
+    kname = (f"sa_group_kernel<{G},{E}> (CDD, {32 // G} chains per warp"
+             + (", 4-bit weights + sub-block summaries)" if nib else ")") if G < 32
              else f"sa_kernel<{E}> (CDD, one warp per chain)")
     # The bound is instruction issue: the kernel does byte-SIMD (one IMAD forms four byte prefixes,
     # one IDP.4A dots four jobs), so the 6n ALGORITHMIC ops per evaluation can run faster than one

@@ -93,7 +93,10 @@ CDD_API int cdd_instance_create(int32_t n, const int32_t *p, const int32_t *alph
 CDD_API int cdd_instance_destroy(cdd_instance *inst);
 /* n, d, sum of p, and flags (bit0: UCDDCP data present, bit1: d >= sum p, bit2: the CDD runs on
  * the generic path, bit3: the UCDDCP runs on the generic path -- its packed record does not fit
- * even where the CDD's does).  Any out may be NULL. */
+ * even where the CDD's does, bit4: the CDD's asynchronous SA at 8 threads x 128 positions per
+ * chain (n in (512, 1024]) uses the small-weight layout -- alpha, beta <= 15 and
+ * max(p) * max(alpha, beta) * 120 < 2^16: 4-bit weights and cached sub-block summaries, same
+ * results).  Any out may be NULL. */
 CDD_API int cdd_instance_query(const cdd_instance *inst, int32_t *n, int64_t *d, int64_t *sum_p,
                        int32_t *flags);
 

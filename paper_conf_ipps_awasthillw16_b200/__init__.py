@@ -151,12 +151,13 @@ class Instance:
         return cls(inst.P, inst.alpha, inst.beta, inst.d, inst.M, inst.gamma, device)
 
     def query(self):
-        """cdd_instance_query: dict(n, d, sum_p, has_ucddcp, unrestricted)."""
+        """cdd_instance_query: dict(n, d, sum_p, has_ucddcp, unrestricted, generic, ucddcp_generic,
+        small_weights)."""
         n, d, sp, fl = C.c_int32(), C.c_int64(), C.c_int64(), C.c_int32()
         _check(_lib.cdd_instance_query(self.handle, C.byref(n), C.byref(d), C.byref(sp), C.byref(fl)))
         return dict(n=n.value, d=d.value, sum_p=sp.value, has_ucddcp=bool(fl.value & 1),
                     unrestricted=bool(fl.value & 2), generic=bool(fl.value & 4),
-                    ucddcp_generic=bool(fl.value & 8))
+                    ucddcp_generic=bool(fl.value & 8), small_weights=bool(fl.value & 16))
 
     @property
     def handle(self):

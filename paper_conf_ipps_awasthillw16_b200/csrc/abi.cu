@@ -333,7 +333,8 @@ int cdd_instance_query(const cdd_instance* I, int32_t* n, int64_t* d, int64_t* s
     if (n) *n = I->n;
     if (d) *d = I->d;
     if (sum_p) *sum_p = I->sum_p;
-    if (flags) *flags = (I->has_ucd ? 1 : 0) | (I->d >= I->sum_p ? 2 : 0) | (I->wide ? 4 : 0) | (I->ucd_wide ? 8 : 0);
+    if (flags) *flags = (I->has_ucd ? 1 : 0) | (I->d >= I->sum_p ? 2 : 0) | (I->wide ? 4 : 0) | (I->ucd_wide ? 8 : 0) |
+                          (I->nib_ok && !I->wide ? 16 : 0);
     return CDD_OK;
 }
 

@@ -848,7 +848,13 @@ __global__ void __launch_bounds__(kGThreads, sag_min_blocks<G, E, UCD, MV>()) sa
             }
             __syncwarp();
             if constexpr (MV == 2) {
-                if (mover) ch.sum()[sidx] = nib_summary(ch, myq & ~15);
+                // the moved sub-blocks' summaries: mover h (lane h < P) joins its half [k0, k0+8)
+                // with lane h + 4's [k0+8, k0+16) (movers sharing a sub-block write equal values)
+                const int h = l & 3;
+                const int hq = h < P ? (int)(((h < 2 ? q01 : q23) >> (16 * (h & 1))) & 0xffffu) : 0;
+                const uint2 part = nib_half(ch, (hq & ~15) | (l & 4 ? 8 : 0));
+                const uint2 other = make_uint2(__shfl_xor_sync(kFull, part.x, 4, G), __shfl_xor_sync(kFull, part.y, 4, G));
+                if (mover) ch.sum()[sidx] = nib_join(part, other);
                 __syncwarp();
             }
             const uint2 tn = ch.tot()[l];

@@ -87,6 +87,36 @@ __device__ __forceinline__ uint2 nib_summary(const GChainNib<G, E>& ch, int k0) 
     return make_uint2(accA | (accB << 16), sA | (sB << 8) | (P << 16));
 }
 
+// Half of a sub-block's summary, positions [k0, k0 + 8) (k0 a multiple of 8), in the same packed
+// format; the summary of [k0, k0 + 16) is nib_join(half at k0, half at k0 + 8).  The kernel splits
+// a mover's recomputation between the mover (lanes 0-3) and lane l ^ 4 of its group.
+template <int G, int E>
+__device__ __forceinline__ uint2 nib_half(const GChainNib<G, E>& ch, int k0) {
+    static_assert(G == 8, "mover lanes 0-3 pair with lanes 4-7 of their group");
+    const uint2 w2 = *reinterpret_cast<const uint2*>(ch.ab() + k0);
+    const uint2 q2 = *reinterpret_cast<const uint2*>(ch.pb() + k0);
+    const uint32_t w[2] = {w2.x, w2.y}, q[2] = {q2.x, q2.y};
+    uint32_t accA = 0, accB = 0, sA = 0, sB = 0, P = 0;
+#pragma unroll
+    for (int j = 0; j < 2; ++j) {
+        const uint32_t a = w[j] & 0x0f0f0f0fu, b = (w[j] >> 4) & 0x0f0f0f0fu;
+        const uint32_t pq = __dp4a(q[j], 0x01010101u, 0u);
+        accA = __dp4a(a * 0x01010100u, q[j], accA) + sA * pq;
+        accB = __dp4a(b * 0x01010100u, q[j], accB) + sB * pq;
+        sA = __dp4a(a, 0x01010101u, sA);
+        sB = __dp4a(b, 0x01010101u, sB);
+        P += pq;
+    }
+    return make_uint2(accA | (accB << 16), sA | (sB << 8) | (P << 16));
+}
+// lo then hi: acc = acc_lo + acc_hi + X_lo * P_hi for both weights (no carry between the 16-bit
+// halves: the joined forms fit 16 bits), the byte sums and P add field-wise
+__device__ __forceinline__ uint2 nib_join(uint2 lo, uint2 hi) {
+    const uint32_t ph = hi.y >> 16;
+    const uint32_t cross = (lo.y & 0xffu) * ph + (((lo.y >> 8) & 0xffu) * ph << 16);
+    return make_uint2(lo.x + hi.x + cross, lo.y + hi.y);
+}
+
 // ---- hooks of boundary_two_level (sa_group.cuh) for this layout
 // level 1: sub-block l of row Ls from its summary
 template <int G, int E>
@@ -94,8 +124,8 @@ __device__ __forceinline__ void bt_level1(const GChainNib<G, E>& ch, int Ls, int
                                           uint32_t& Sb1, uint32_t& dot) {
     const uint2 s = ch.sum()[l * G + Ls];
     Pb1 = s.y >> 16;
-    Sb1 = (s.y & 0xffu) + ((s.y >> 8) & 0xffu);
-    dot = (s.x & 0xffffu) + (s.x >> 16);
+    Sb1 = __dp4a(s.y, 0x0101u, 0u);       // A_b + B_b
+    dot = __dp2a_lo(s.x, 0x0101u, 0u);    // acc_A + acc_B
 }
 // level 2: L2 <= 4 consecutive positions from e (row-relative) of row Ls as alpha|beta<<8 pair
 // words and a P word
@@ -142,15 +172,17 @@ __device__ __forceinline__ int32_t gchain_eval_nib(const GChainNib<G, E>& ch, in
     const uint32_t key = ((uint32_t)min(thr, 0xffff) << 16) | 0xffffu;
     const int32_t corr = boundary_two_level<G, E>(ch, l, gbase, Ls, Lk, d, PbS, thr, key, quad);
     // F(C_{m'}): the row form of x = alpha (lanes left of Ls) or beta from the 8 summaries
+    // per sub-block: IDP.2A picks and adds acc_A or acc_B (16-bit halves x (1, 0) / (0, 1)),
+    // IDP.4A picks and adds A_b or B_b, one IMAD for Xbefore * P_b
     const bool amode = l < Ls;
-    const uint32_t asel = amode ? 0x4410u : 0x4432u, xsel = amode ? 0x4440u : 0x4441u;
+    const uint32_t asel = amode ? 0x0001u : 0x0100u, xsel = amode ? 0x0001u : 0x0100u;
     const uint2* srow = ch.sum() + l;
     uint32_t acc = 0, xb = 0;
 #pragma unroll
     for (int b = 0; b < E / 16; ++b) {
         const uint2 s = srow[b * G];
-        acc += __byte_perm(s.x, 0u, asel) + xb * (s.y >> 16);
-        xb += __byte_perm(s.y, 0u, xsel);
+        acc = __dp2a_lo(s.x, asel, acc) + xb * (s.y >> 16);
+        xb = __dp4a(s.y, xsel, xb);
     }
     const int32_t base = amode ? Ab : (Btot - Bb);
     const int32_t contrib = base * (int32_t)tP + (amode ? (int32_t)acc : -(int32_t)acc) + corr;

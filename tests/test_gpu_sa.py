@@ -451,7 +451,7 @@ def test_nibble_layout_trace_parity(lib, n, kw, move, pert):
     chains, steps, seed = 48, 150, 77 + n
     ins, res, (pen, perm, gid), pr, p, T0 = _run_both(lib, inst, "cdd", chains, steps, seed, samples=300,
                                                      move=move, pert=pert, lanes=8)
-    assert lib.sa_layout(ins, chains, lanes=8) == (8, 128)
+    assert lib.sa_layout(ins, chains, lanes=8) == (8, 128) and ins.query()["small_weights"]
     tr = res["trace"].cpu().numpy()
     for c in range(chains):
         ref = oracle.sa_chain(pr, p, T0, c, trace=True)
@@ -485,3 +485,14 @@ def test_nibble_layout_full_grid_and_balanced(lib):
         for c in list(range(0, chains, 997)) + [chains - 1]:
             ref = oracle.sa_chain(pr, p, 500.0, c)
             assert (cb[c], cf[c]) == (ref["E_best"], ref["E_final"]), c
+
+
+def test_small_weights_flag(lib):
+    # cdd_instance_query bit4 follows the layout's conditions (alpha, beta <= 15, pmax * 15 * 120 < 2^16)
+    for kw, want in [(dict(p=(1, 20), alpha=(1, 10), beta=(1, 15)), True),
+                     (dict(p=(36, 36), alpha=(15, 15), beta=(1, 1)), True),
+                     (dict(p=(37, 37), alpha=(15, 15), beta=(1, 1)), False),
+                     (dict(p=(1, 20), alpha=(1, 16), beta=(1, 15)), False),
+                     (dict(p=(1, 20), alpha=(1, 10), beta=(1, 16)), False)]:
+        inst = gen.ranged_instance(600, 2, h=0.5, **kw)
+        assert lib.Instance.from_gen(inst).query()["small_weights"] == want, kw
