@@ -200,6 +200,7 @@ struct GroupCfg {
 CDD_SAG_DECL(sag_cdd)
 CDD_SAG_DECL(sag_cdd_tr)
 CDD_SAG_DECL(sag_cdd_nib)
+CDD_SAG_SYNC_DECL(sag_cdd_nib)
 CDD_SAG_DECL(sag_cdd_nib_tr)
 CDD_SAG_DECL(sag_ucd)
 CDD_SAG_DECL(sag_ucd_tr)

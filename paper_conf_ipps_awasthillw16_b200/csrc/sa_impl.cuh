@@ -1239,10 +1239,10 @@ __global__ void sync_level_finalize(unsigned long long* keys, const int16_t* slo
 // chain holding s^min_{j-1} (exactly what gchain_init writes for it, zero padding elsewhere).
 // After the cross-GPU exchange smin holds the global s^min, so the image is built here, not in
 // sync_level_finalize.
-template <int G, int E, bool UCD>
+template <int G, int E, bool UCD, int MV>
 __global__ void sync_level_prepare(double* T, double mu, unsigned long long* keys, const int16_t* smin,
                                    int n, ChainTables tb, uint8_t* image, int16_t* ids, int* err) {
-    using C = GChain<G, E, UCD>;
+    using C = SagChain<G, E, UCD, MV>;
     constexpr int NP = C::NP;
     if (threadIdx.x == 0) {
         *T = __dmul_rn(*T, mu);
@@ -1263,18 +1263,37 @@ __global__ void sync_level_prepare(double* T, double mu, unsigned long long* key
         ids[k] = (int16_t)j;
         const bool v = k < n;
         const uint32_t ab = v ? tb.ab16[j] : 0u;
-        ch.pb()[C::pb_b(k)] = v ? tb.p[j] : (uint8_t)0;
-        if constexpr (UCD) {
+        if constexpr (MV == 2) {  // nibble layout (sa_nib.cuh)
+            ch.ab()[k] = (uint8_t)((ab & 15u) | ((ab >> 4) & 0xf0u));
+            ch.pb()[k] = v ? tb.p[j] : (uint8_t)0;
+        } else if constexpr (UCD) {
+            ch.pb()[C::pb_b(k)] = v ? tb.p[j] : (uint8_t)0;
             ch.ab()[C::ab_h(k)] = (uint16_t)ab;
             ch.xb()[C::pb_b(k)] = v ? tb.x[j] : (uint8_t)0;
             ch.gh()[C::gh_h(k)] = v ? tb.g[j] : (uint16_t)0;
         } else {
+            ch.pb()[C::pb_b(k)] = v ? tb.p[j] : (uint8_t)0;
             ch.a8()[C::rb(k)] = (uint8_t)ab;
             ch.b8()[C::rb(k)] = (uint8_t)(ab >> 8);
         }
     }
     __syncthreads();
-    if (threadIdx.x < G) ch.tot()[threadIdx.x] = gchain_lane_totals(ch, (int)threadIdx.x);
+    if constexpr (MV == 2) {
+        if (threadIdx.x < G) {  // the lane row's sub-block summaries and totals, as gchain_init
+            const int l = (int)threadIdx.x;
+            uint32_t tA = 0, tB = 0, tP = 0;
+            for (int b = 0; b < C::NSB; ++b) {
+                const uint2 sm = nib_summary(ch, l * E + 16 * b);
+                ch.sum()[b * G + l] = sm;
+                tA += sm.y & 0xffu;
+                tB += (sm.y >> 8) & 0xffu;
+                tP += sm.y >> 16;
+            }
+            ch.tot()[l] = make_uint2(tA | (tB << 16), tP);
+        }
+    } else {
+        if (threadIdx.x < G) ch.tot()[threadIdx.x] = gchain_lane_totals(ch, (int)threadIdx.x);
+    }
     __syncthreads();
     for (int i = threadIdx.x; i < C::BYTES / 16; i += blockDim.x)
         reinterpret_cast<int4*>(image)[i] = reinterpret_cast<const int4*>(buf)[i];
@@ -1297,7 +1316,7 @@ SyncWs sync_layout(const Instance& I, const SaLaunch& p) {
     w.keys_off = align_up(w.T_off + sizeof(double));
     w.smin_off = align_up(w.keys_off + 2 * sizeof(unsigned long long));
     w.image_off = align_up(w.smin_off + (size_t)NP * sizeof(int16_t));
-    w.ids_off = align_up(w.image_off + (size_t)GChain<G, E, UCD>::BYTES);
+    w.ids_off = align_up(w.image_off + (size_t)SagChain<G, E, UCD, MV>::BYTES);
     w.total = align_up(w.ids_off + (size_t)NP * sizeof(int16_t));
     return w;
 }
@@ -1332,7 +1351,7 @@ cudaError_t sag_sync_level(Instance& I, const SaLaunch& p, int64_t j, int64_t* l
         e = cudaMemsetAsync(keys, 0xff, 2 * sizeof(unsigned long long), s);
         if (e != cudaSuccess) return e;
     } else {
-        sync_level_prepare<G, E, UCD><<<1, 256, 0, s>>>(T, p.mu, keys, smin, I.n, tables(I, UCD),
+        sync_level_prepare<G, E, UCD, MV><<<1, 256, 0, s>>>(T, p.mu, keys, smin, I.n, tables(I, UCD),
                                                         base + w.image_off,
                                                         reinterpret_cast<int16_t*>(base + w.ids_off), I.err);
         e = cudaGetLastError();
@@ -1451,6 +1470,24 @@ int pow2_at_least(int c) {
     cudaError_t NAME##_run(Instance& I, const SaLaunch& p, GroupCfg cfg, void* ws, cudaStream_t s) { \
         return cfg.G == 8 && cfg.E == 128 ? sag_impl<8, 128, false, TR, 2>(I, p, ws, s)           \
                                           : cudaErrorInvalidValue;                               \
+    }
+// ... and its synchronous-SA levels
+#define CDD_SAG_NIB_SYNC_VARIANT(NAME)                                                            \
+    size_t NAME##_sync_ws(const Instance& I, const SaLaunch& p, GroupCfg cfg) {                  \
+        return cfg.G == 8 && cfg.E == 128 ? sync_layout<8, 128, false, 2>(I, p).total : 0;       \
+    }                                                                                            \
+    cudaError_t NAME##_sync_level(Instance& I, const SaLaunch& p, GroupCfg cfg, int64_t j,       \
+                                  int64_t* level_min, void* ws, cudaStream_t s) {                \
+        return cfg.G == 8 && cfg.E == 128 ? sag_sync_level<8, 128, false, 2>(I, p, j, level_min, ws, s) \
+                                          : cudaErrorInvalidValue;                               \
+    }                                                                                            \
+    void NAME##_sync_ptrs(const Instance& I, const SaLaunch& p, GroupCfg cfg, void* ws,          \
+                          unsigned long long** key, int16_t** perm) {                            \
+        const SyncWs w = sync_layout<8, 128, false, 2>(I, p);                                    \
+        (void)cfg;                                                                               \
+        uint8_t* base = static_cast<uint8_t*>(ws);                                               \
+        *key = reinterpret_cast<unsigned long long*>(base + w.keys_off) + 1;                     \
+        *perm = reinterpret_cast<int16_t*>(base + w.smin_off);                                   \
     }
 
 #define CDD_SAG_T0_VARIANT(NAME, UCD)                                                             \

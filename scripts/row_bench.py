@@ -112,6 +112,21 @@ def main():
         out("A9-A11", f"SA {prob} n={n}, {C} chains x {S} steps", ev / dt, "evals/s",
             ops * n * ev / dt / 1e12, alu, "Tint-op/s", f"{ops}n algorithmic int ops per evaluation")
 
+    # the headline SA with the byte-row layout (CDD_SA_NO_NIB=1: no 4-bit weights, no sub-block
+    # summaries) for comparison with the small-weight layout the row above uses
+    if want("A9"):
+        C, S = 65536, 1000
+        os.environ["CDD_SA_NO_NIB"] = "1"
+        try:
+            t0 = cdd.sa_t0(ic, seed=1, samples=T0)
+            ws = cdd.sa_run(ic, C, S, seed=1, T0_dev=t0)["workspace"]
+            dt = timed(lambda r=0: cdd.sa_run(ic, C, S, seed=1, T0_dev=t0, workspace=ws), reps=3)
+        finally:
+            del os.environ["CDD_SA_NO_NIB"]
+        ev = C * (S + 1)
+        out("A9-A11", f"SA cdd n={n} byte-row layout (CDD_SA_NO_NIB=1), {C} chains x {S} steps", ev / dt,
+            "evals/s", 6 * n * ev / dt / 1e12, alu, "Tint-op/s", "6n algorithmic int ops per evaluation")
+
     # F2 synchronous SA
     C, M, L = 65536, 50, 20
     if want("F2"):
