@@ -826,7 +826,10 @@ __global__ void __launch_bounds__(kGThreads, sag_min_blocks<G, E, UCD, MV>()) sa
             const int myq = mover ? (int)(((l < 2 ? q01 : q23) >> (16 * (l & 1))) & 0xffffu) : 0;
             const uint2 old_v = pos_read<G, E, UCD>(ch, myq);
             // nibble layout: the summary of the mover's sub-block (every mover reads before any
-            // writes; movers sharing a sub-block write the same values)
+            // writes).  Movers sharing a sub-block store the same value with the same warp
+            // instruction (the join below, the restore on rejection), where CUDA keeps exactly one
+            // of the lanes' writes -- so the result is that value.  (Electing one writer per
+            // sub-block was measured 2.5 % slower.)
             uint2 old_s = make_uint2(0u, 0u);
             int sidx = 0;
             if constexpr (MV == 2) {

@@ -29,6 +29,16 @@ for n in (7, 50, 100, 200, 500, 777, 1000):
     if n >= 2:
         cdd.dpso_run(u, 64, 5, problem="ucddcp", seed=2)
     cdd.cdd_check(u)
+# the small-weight SA layout (csrc/sa_nib.cuh: 4-bit weights, sub-block summaries, lane-pair
+# recomputation) at G = 8, E = 128: every move of <= 4 positions, synchronous levels
+for n in (600, 1000):
+    ins = cdd.Instance.from_gen(gen.cdd_instance(n, 3, 0.6))
+    assert ins.query()["small_weights"]
+    for mv, pert in (("pert_fy", 4), ("swap", 2), ("window", 4), ("pert_fy", 3)):
+        cdd.sa_run(ins, 64, 12, seed=5, t0_samples=100, lanes=8, move=mv, pert=pert)
+    cdd.sa_run(ins, 64, 12, seed=5, t0_samples=100, lanes=8, trace=True)
+    cdd.SaSync(ins, 64, 6, 3, seed=3, t0_samples=100, lanes=8).run()
+    cdd.cdd_check(ins)
 # balanced SA schedule (chains split between warps, state handed over): more chains than slots
 ins = cdd.Instance.from_gen(gen.cdd_instance(120, 2, 0.4))
 cdd.sa_run(ins, 15000, 9, seed=4, T0=900.0, lanes=8)
