@@ -25,7 +25,9 @@ def lib():
     (60, 100, 200, "cdd", 32, False),
     (300, 2000, 120, "cdd", 0, False),     # group layout
     (300, 70, 120, "cdd", 8, True),
-    (1000, 1200, 60, "cdd", 0, False),    # the headline layout (8 lanes x 128)
+    (1000, 1200, 60, "cdd", 0, False),    # automatic layout (16 lanes x 64 at 1200 chains)
+    (1000, 300, 60, "cdd", 8, False),     # the headline layout: 8 lanes x 128, small-weight records
+    (1000, 300, 60, "cdd", 8, True),
     (200, 300, 100, "ucddcp", 0, False),
     (200, 300, 100, "ucddcp", 32, True),
 ])
