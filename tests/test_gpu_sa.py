@@ -434,7 +434,8 @@ def test_balanced_schedule_every_chain(lib, problem, n, chains, steps):
 
 # The nibble layout with sub-block summaries (csrc/sa_nib.cuh): CDD with alpha, beta <= 15 and
 # pmax * max(alpha, beta) * 120 < 2^16 at G = 8, E = 128 (n in (512, 1024]).  Every move of <= 4
-# positions, traced chain by chain against the oracle, and the same run with the byte-row layout
+# positions (insertion keeps the byte rows at this layout: the same check covers it), traced chain
+# by chain against the oracle, and the same run with the byte-row layout
 # (CDD_SA_NO_NIB=1) must give the identical trace.  The instances put the 16-bit sub-block forms
 # at their limit (p up to 36 with weights 15: 36 * 15 * 120 = 64800) and n off the sub-block grid.
 NIB = [
@@ -445,7 +446,7 @@ NIB = [
 
 
 @pytest.mark.parametrize("n,kw", NIB)
-@pytest.mark.parametrize("move,pert", [("pert_fy", 4), ("pert_fy", 3), ("swap", 2), ("window", 4)])
+@pytest.mark.parametrize("move,pert", [("pert_fy", 4), ("pert_fy", 3), ("swap", 2), ("window", 4), ("insert", 4)])
 def test_nibble_layout_trace_parity(lib, n, kw, move, pert):
     inst = gen.ranged_instance(n, 5, **kw)
     chains, steps, seed = 48, 150, 77 + n
