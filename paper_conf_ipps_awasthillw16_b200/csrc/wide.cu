@@ -156,6 +156,63 @@ __device__ __forceinline__ WideSplit wide_split(const WideTab& T, int n, int t, 
 // wholly before the due date D contributes A (D - C_start) - DA, one wholly after it
 // B (C_start - D) + DB; only the thread whose segment holds D walks it again (and the owner of
 // k0, for C_{k0}) -- the split F(C) = F(C_m') + integral of the fast kernels.
+// Warp inclusive scan of int64 values (one warp group, TH = 32).
+__device__ __forceinline__ long long warp_incl_scan64(long long x, int lane) {
+#pragma unroll
+    for (int off = 1; off < 32; off <<= 1) {
+        const long long y = __shfl_up_sync(kFull, x, off);
+        if (lane >= off) x += y;
+    }
+    return x;
+}
+
+// One warp per sequence: the two segment walks of wide_eval_cdd (C_{k0} in the owner's segment,
+// the objective over the segment holding D) spread over the 32 lanes, 32 positions per round, with
+// warp scans of P and alpha + beta instead of one thread walking S positions.
+template <class IdAt>
+__device__ __forceinline__ long long wide_walk_k0_warp(const WideTab& T, int ka, int kb, long long s0, long long c0,
+                                                       long long Btot, int lane, IdAt&& id_at) {
+    long long cc = 0;
+    for (int k1 = ka; k1 < kb; k1 += 32) {  // warp-uniform
+        const int k = k1 + lane;
+        long long p = 0, w = 0;
+        if (k < kb) {
+            const int4 r = __ldg(T.w0 + id_at(k));
+            p = r.x;
+            w = (long long)r.y + r.z;
+        }
+        const long long ip = warp_incl_scan64(p, lane), iw = warp_incl_scan64(w, lane);
+        // S_k (exclusive) <= Btot: a prefix of the positions; the last one's inclusive C
+        const unsigned m = __ballot_sync(kFull, k < kb && s0 + iw - w <= Btot);
+        if (m) cc = __shfl_sync(kFull, c0 + ip, 31 - __clz(m));
+        if (!(m >> 31)) break;  // the prefix ended inside this round (or the segment did)
+        s0 += __shfl_sync(kFull, iw, 31);
+        c0 += __shfl_sync(kFull, ip, 31);
+    }
+    return cc;
+}
+
+template <class IdAt>
+__device__ __forceinline__ long long wide_walk_D_warp(const WideTab& T, int ka, int kb, long long c0, long long D,
+                                                      int lane, IdAt&& id_at) {
+    long long z = 0;
+    for (int k1 = ka; k1 < kb; k1 += 32) {
+        const int k = k1 + lane;
+        long long p = 0, a = 0, b = 0;
+        if (k < kb) {
+            const int4 r = __ldg(T.w0 + id_at(k));
+            p = r.x;
+            a = r.y;
+            b = r.z;
+        }
+        const long long ip = warp_incl_scan64(p, lane);
+        const long long c = c0 + ip;
+        if (k < kb) z += D > c ? a * (D - c) : b * (c - D);
+        c0 += __shfl_sync(kFull, ip, 31);
+    }
+    return z;  // this lane's share
+}
+
 template <int TH, class IdAt>
 __device__ __forceinline__ long long wide_eval_cdd(const WideTab& T, int n, long long d, int t, IdAt&& id_at,
                                                    long long* sm) {
@@ -174,10 +231,14 @@ __device__ __forceinline__ long long wide_eval_cdd(const WideTab& T, int n, long
     const long long Pex = wgroup_excl_scan<TH>(Pt, Ptot, sm);
     const long long Aex = wgroup_excl_scan<TH>(At, Atot, sm);
     const long long Bex = wgroup_excl_scan<TH>(Bt, Btot, sm);
-    // k0 = max{k : S_k <= Btot} (a prefix): the owner walks its segment for C_{k0}
+    // k0 = max{k : S_k <= Btot} (a prefix): the owner's segment is walked for C_{k0}
     const int own = wgroup_max<TH>((ka < kb && Aex + Bex <= Btot) ? t : 0, sm);
     long long cc = 0;
-    if (t == own) {
+    if constexpr (TH == 32) {
+        const int oka = min(n, own * S), okb = min(n, oka + S);
+        cc = wide_walk_k0_warp(T, oka, okb, __shfl_sync(kFull, Aex + Bex, own), __shfl_sync(kFull, Pex, own),
+                               Btot, t, id_at);
+    } else if (t == own) {
         long long s = Aex + Bex, c = Pex;
         for (int k = ka; k < kb; ++k) {
             const int4 r = __ldg(T.w0 + id_at(k));
@@ -186,20 +247,23 @@ __device__ __forceinline__ long long wide_eval_cdd(const WideTab& T, int n, long
             s += (long long)r.y + r.z;
         }
     }
-    const long long D = min(wgroup_bcast<TH>(cc, own, sm), d);
+    const long long D = TH == 32 ? min(cc, d) : min(wgroup_bcast<TH>(cc, own, sm), d);
     long long z = 0;
-    if (ka < kb) {
-        if (Pex + Pt <= D) {
-            z = At * (D - Pex) - DA;
-        } else if (Pex >= D) {
-            z = Bt * (Pex - D) + DB;
-        } else {  // the segment that holds D
-            long long c = Pex;
-            for (int k = ka; k < kb; ++k) {
-                const int4 r = __ldg(T.w0 + id_at(k));
-                c += r.x;
-                z += D > c ? (long long)r.y * (D - c) : (long long)r.z * (c - D);
-            }
+    const bool holds = ka < kb && Pex < D && Pex + Pt > D;  // the segment that holds D (at most one)
+    if (ka < kb && !holds) z = Pex + Pt <= D ? At * (D - Pex) - DA : Bt * (Pex - D) + DB;
+    if constexpr (TH == 32) {
+        const unsigned hm = __ballot_sync(kFull, holds);
+        if (hm) {
+            const int th = __ffs(hm) - 1;
+            const int hka = min(n, th * S), hkb = min(n, hka + S);
+            z += wide_walk_D_warp(T, hka, hkb, __shfl_sync(kFull, Pex, th), D, t, id_at);
+        }
+    } else if (holds) {
+        long long c = Pex;
+        for (int k = ka; k < kb; ++k) {
+            const int4 r = __ldg(T.w0 + id_at(k));
+            c += r.x;
+            z += D > c ? (long long)r.y * (D - c) : (long long)r.z * (c - D);
         }
     }
     return wgroup_sum<TH>(z, sm);
