@@ -442,6 +442,11 @@ NIB = [
     (1000, dict(p=(1, 20), alpha=(1, 10), beta=(1, 15), h=0.4)),
     (777, dict(p=(30, 36), alpha=(14, 15), beta=(13, 15), h=0.6)),
     (530, dict(p=(1, 36), alpha=(0, 15), beta=(0, 15), h=0.2)),
+    # edges: n just above E = 64 (lanes 5-7 hold padding), n = 1024 (no padding), zero weights,
+    # d = 0 and d >= sum p, every value at the layout's limit (acc = 36 * 15 * 120 = 64800)
+    (513, dict(p=(1, 20), alpha=(0, 0), beta=(1, 15), h=0.0)),
+    (1024, dict(p=(1, 20), alpha=(1, 15), beta=(0, 0), h=1.2)),
+    (1024, dict(p=(36, 36), alpha=(15, 15), beta=(15, 15), h=0.5)),
 ]
 
 
