@@ -382,7 +382,7 @@ __device__ void gchain_init(const GChainNib<G, E>& ch, int16_t* cur, int n, uint
     uint32_t tA = 0, tB = 0, tP = 0;
 #pragma unroll
     for (int b = 0; b < C::NSB; ++b) {
-        const uint2 sm = nib_summary(ch, l * E + 16 * b);
+        const uint2 sm = nib_summary(ch, l * E + C::SB * b);
         ch.sum()[b * G + l] = sm;
         tA += sm.y & 0xffu;
         tB += (sm.y >> 8) & 0xffu;
@@ -855,7 +855,7 @@ __global__ void __launch_bounds__(kGThreads, sag_min_blocks<G, E, UCD, MV>()) sa
                 // with lane h + 4's [k0+8, k0+16) (movers sharing a sub-block write equal values)
                 const int h = l & 3;
                 const int hq = h < P ? (int)(((h < 2 ? q01 : q23) >> (16 * (h & 1))) & 0xffffu) : 0;
-                const uint2 part = nib_half(ch, (hq & ~15) | (l & 4 ? 8 : 0));
+                const uint2 part = nib_half(ch, (hq & ~(C::SB - 1)) | (l & 4 ? C::SB / 2 : 0));
                 const uint2 other = make_uint2(__shfl_xor_sync(kFull, part.x, 4, G), __shfl_xor_sync(kFull, part.y, 4, G));
                 if (mover) ch.sum()[sidx] = nib_join(part, other);
                 __syncwarp();
@@ -1286,7 +1286,7 @@ __global__ void sync_level_prepare(double* T, double mu, unsigned long long* key
             const int l = (int)threadIdx.x;
             uint32_t tA = 0, tB = 0, tP = 0;
             for (int b = 0; b < C::NSB; ++b) {
-                const uint2 sm = nib_summary(ch, l * E + 16 * b);
+                const uint2 sm = nib_summary(ch, l * E + C::SB * b);
                 ch.sum()[b * G + l] = sm;
                 tA += sm.y & 0xffu;
                 tB += (sm.y >> 8) & 0xffu;
@@ -1468,26 +1468,31 @@ int pow2_at_least(int c) {
 // The nibble-layout variant (MV = 2, sa_nib.cuh): CDD, G = 8, E = 128 only.
 #define CDD_SAG_NIB_VARIANT(NAME, TR)                                                             \
     size_t NAME##_ws(const Instance& I, const SaLaunch& p, GroupCfg cfg) {                       \
-        return cfg.G == 8 && cfg.E == 128 ? sag_ws<8, 128, false, TR, 2>(I, p) : 0;              \
+        if (cfg.G == 8 && cfg.E == 128) return sag_ws<8, 128, false, TR, 2>(I, p);               \
+        if (cfg.G == 8 && cfg.E == 64) return sag_ws<8, 64, false, TR, 2>(I, p);                 \
+        return 0;                                                                                \
     }                                                                                            \
     cudaError_t NAME##_run(Instance& I, const SaLaunch& p, GroupCfg cfg, void* ws, cudaStream_t s) { \
-        return cfg.G == 8 && cfg.E == 128 ? sag_impl<8, 128, false, TR, 2>(I, p, ws, s)           \
-                                          : cudaErrorInvalidValue;                               \
+        if (cfg.G == 8 && cfg.E == 128) return sag_impl<8, 128, false, TR, 2>(I, p, ws, s);      \
+        if (cfg.G == 8 && cfg.E == 64) return sag_impl<8, 64, false, TR, 2>(I, p, ws, s);        \
+        return cudaErrorInvalidValue;                                                            \
     }
 // ... and its synchronous-SA levels
 #define CDD_SAG_NIB_SYNC_VARIANT(NAME)                                                            \
     size_t NAME##_sync_ws(const Instance& I, const SaLaunch& p, GroupCfg cfg) {                  \
-        return cfg.G == 8 && cfg.E == 128 ? sync_layout<8, 128, false, 2>(I, p).total : 0;       \
+        if (cfg.G == 8 && cfg.E == 128) return sync_layout<8, 128, false, 2>(I, p).total;        \
+        if (cfg.G == 8 && cfg.E == 64) return sync_layout<8, 64, false, 2>(I, p).total;          \
+        return 0;                                                                                \
     }                                                                                            \
     cudaError_t NAME##_sync_level(Instance& I, const SaLaunch& p, GroupCfg cfg, int64_t j,       \
                                   int64_t* level_min, void* ws, cudaStream_t s) {                \
-        return cfg.G == 8 && cfg.E == 128 ? sag_sync_level<8, 128, false, 2>(I, p, j, level_min, ws, s) \
-                                          : cudaErrorInvalidValue;                               \
+        if (cfg.G == 8 && cfg.E == 128) return sag_sync_level<8, 128, false, 2>(I, p, j, level_min, ws, s); \
+        if (cfg.G == 8 && cfg.E == 64) return sag_sync_level<8, 64, false, 2>(I, p, j, level_min, ws, s); \
+        return cudaErrorInvalidValue;                                                            \
     }                                                                                            \
     void NAME##_sync_ptrs(const Instance& I, const SaLaunch& p, GroupCfg cfg, void* ws,          \
                           unsigned long long** key, int16_t** perm) {                            \
-        const SyncWs w = sync_layout<8, 128, false, 2>(I, p);                                    \
-        (void)cfg;                                                                               \
+        const SyncWs w = cfg.E == 128 ? sync_layout<8, 128, false, 2>(I, p) : sync_layout<8, 64, false, 2>(I, p); \
         uint8_t* base = static_cast<uint8_t*>(ws);                                               \
         *key = reinterpret_cast<unsigned long long*>(base + w.keys_off) + 1;                     \
         *perm = reinterpret_cast<int16_t*>(base + w.smin_off);                                   \

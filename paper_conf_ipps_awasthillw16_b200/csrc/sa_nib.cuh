@@ -16,9 +16,11 @@
 // the alpha+beta prefix is acc_A + acc_B.
 //
 // Applies when alpha, beta <= 15 and pmax * max(alpha, beta) * 120 < 2^16 (acc_b fits 16 bits;
-// 120 = sum of the in-block prefix counts 0..15), n in (512, 1024] (G = 8, E = 128): the
-// OR-library ranges (p <= 20, alpha <= 10, beta <= 15) at BASELINE config 5.  The records take 2
-// bytes per position instead of 3 and no padding, so 5 CTAs (20 warps) fit an SM instead of 4.
+// 120 = sum of the in-block prefix counts 0..15), at G = 8 lanes per chain with E = 128 (n in
+// (512, 1024], 16-position sub-blocks) or E = 64 (n in (256, 512], 8-position sub-blocks; one
+// sub-block per lane of the boundary's level 1 either way): the OR-library ranges (p <= 20,
+// alpha <= 10, beta <= 15), e.g. BASELINE config 5.  The records take 2 bytes per position
+// instead of 3 and no padding, so at n = 1000 5 CTAs (20 warps) fit an SM instead of 4.
 // The arithmetic is exactly the evaluator of sa_group.cuh: same penalties, same trajectories.
 #pragma once
 #include <cuda_runtime.h>
@@ -34,7 +36,8 @@ struct GChainNib {
     // type for every (G, E) of the byte-row layout too)
     static constexpr int NP = G * E;
     static constexpr int SPR = E / G;          // boundary elements per lane (= sub-block length)
-    static constexpr int NSB = E / 16;         // sub-blocks per lane row (= G)
+    static constexpr int SB = E / G;           // positions per sub-block (16 at E = 128, 8 at E = 64)
+    static constexpr int NSB = E / SB;         // sub-blocks per lane row (= G)
     static constexpr int OFF_P = NP, OFF_S = 2 * NP, OFF_T = 2 * NP + 8 * G * NSB;
     // chains are BYTES apart: BYTES % 128 == 64 puts the summaries of a warp's even and odd chains
     // in opposite bank halves (the aggregation's LDS.64 then takes the minimum two wavefronts)
@@ -48,7 +51,7 @@ struct GChainNib {
     //   .x = acc_A | acc_B << 16,  .y = A_b | B_b << 8 | P_b << 16
     __device__ __forceinline__ uint2* sum() const { return reinterpret_cast<uint2*>(base + OFF_S); }
     __device__ __forceinline__ uint2* tot() const { return reinterpret_cast<uint2*>(base + OFF_T); }
-    static __device__ __forceinline__ int sidx(int k) { return ((k % E) / 16) * G + k / E; }
+    static __device__ __forceinline__ int sidx(int k) { return ((k % E) / SB) * G + k / E; }
 };
 
 // u0 = alpha | beta << 8 | P << 16 (the shuffle / lane-total format of pos_read)
@@ -63,19 +66,26 @@ __device__ __forceinline__ void nib_write(const GChainNib<G, E>& ch, int k, uint
     ch.pb()[k] = (uint8_t)(v >> 16);
 }
 
-// Summary of the 16 positions [k0, k0 + 16) (k0 a multiple of 16): the quad form of the SA pass
-// on x = alpha and x = beta (byte-wise prefixes of three 4-bit weights fit a byte).
-template <int G, int E>
-__device__ __forceinline__ uint2 nib_summary(const GChainNib<G, E>& ch, int k0) {
-    using C = GChainNib<G, E>;
-    static_assert(E == 16 * G, "one 16-position sub-block per lane of the boundary row's level 1");
-    static_assert(2 * C::NP + 16 * G <= C::BYTES, "FY staging (ids + Philox words) must fit");
-    const uint4 w4 = *reinterpret_cast<const uint4*>(ch.ab() + k0);
-    const uint4 q4 = *reinterpret_cast<const uint4*>(ch.pb() + k0);
-    const uint32_t w[4] = {w4.x, w4.y, w4.z, w4.w}, q[4] = {q4.x, q4.y, q4.z, q4.w};
+// Summary of the Q quads of positions [k0, k0 + 4Q) (k0 a multiple of 4Q): the quad form of the SA
+// pass on x = alpha and x = beta (byte-wise prefixes of three 4-bit weights fit a byte).
+template <int Q>
+__device__ __forceinline__ uint2 nib_quads(const uint8_t* ab, const uint8_t* pb) {
+    uint32_t w[Q], q[Q];
+    if constexpr (Q == 4) {
+        const uint4 w4 = *reinterpret_cast<const uint4*>(ab), q4 = *reinterpret_cast<const uint4*>(pb);
+        w[0] = w4.x; w[1] = w4.y; w[2] = w4.z; w[3] = w4.w;
+        q[0] = q4.x; q[1] = q4.y; q[2] = q4.z; q[3] = q4.w;
+    } else if constexpr (Q == 2) {
+        const uint2 w2 = *reinterpret_cast<const uint2*>(ab), q2 = *reinterpret_cast<const uint2*>(pb);
+        w[0] = w2.x; w[1] = w2.y;
+        q[0] = q2.x; q[1] = q2.y;
+    } else {
+        w[0] = *reinterpret_cast<const uint32_t*>(ab);
+        q[0] = *reinterpret_cast<const uint32_t*>(pb);
+    }
     uint32_t accA = 0, accB = 0, sA = 0, sB = 0, P = 0;
 #pragma unroll
-    for (int j = 0; j < 4; ++j) {
+    for (int j = 0; j < Q; ++j) {
         const uint32_t a = w[j] & 0x0f0f0f0fu, b = (w[j] >> 4) & 0x0f0f0f0fu;
         const uint32_t pq = __dp4a(q[j], 0x01010101u, 0u);
         accA = __dp4a(a * 0x01010100u, q[j], accA) + sA * pq;
@@ -87,27 +97,22 @@ __device__ __forceinline__ uint2 nib_summary(const GChainNib<G, E>& ch, int k0) 
     return make_uint2(accA | (accB << 16), sA | (sB << 8) | (P << 16));
 }
 
-// Half of a sub-block's summary, positions [k0, k0 + 8) (k0 a multiple of 8), in the same packed
-// format; the summary of [k0, k0 + 16) is nib_join(half at k0, half at k0 + 8).  The kernel splits
-// a mover's recomputation between the mover (lanes 0-3) and lane l ^ 4 of its group.
+// Summary of sub-block [k0, k0 + SB) (k0 a multiple of SB).
+template <int G, int E>
+__device__ __forceinline__ uint2 nib_summary(const GChainNib<G, E>& ch, int k0) {
+    using C = GChainNib<G, E>;
+    static_assert(C::SB == 16 || C::SB == 8, "16- or 8-position sub-blocks, one per lane of the boundary's level 1");
+    static_assert(2 * C::NP + 16 * G <= C::BYTES, "FY staging (ids + Philox words) must fit");
+    return nib_quads<C::SB / 4>(ch.ab() + k0, ch.pb() + k0);
+}
+
+// Half of a sub-block's summary, positions [k0, k0 + SB/2) (k0 a multiple of SB/2), in the same
+// packed format; the summary of the sub-block is nib_join(half at k0, half at k0 + SB/2).  The
+// kernel splits a mover's recomputation between the mover (lanes 0-3) and lane l ^ 4 of its group.
 template <int G, int E>
 __device__ __forceinline__ uint2 nib_half(const GChainNib<G, E>& ch, int k0) {
     static_assert(G == 8, "mover lanes 0-3 pair with lanes 4-7 of their group");
-    const uint2 w2 = *reinterpret_cast<const uint2*>(ch.ab() + k0);
-    const uint2 q2 = *reinterpret_cast<const uint2*>(ch.pb() + k0);
-    const uint32_t w[2] = {w2.x, w2.y}, q[2] = {q2.x, q2.y};
-    uint32_t accA = 0, accB = 0, sA = 0, sB = 0, P = 0;
-#pragma unroll
-    for (int j = 0; j < 2; ++j) {
-        const uint32_t a = w[j] & 0x0f0f0f0fu, b = (w[j] >> 4) & 0x0f0f0f0fu;
-        const uint32_t pq = __dp4a(q[j], 0x01010101u, 0u);
-        accA = __dp4a(a * 0x01010100u, q[j], accA) + sA * pq;
-        accB = __dp4a(b * 0x01010100u, q[j], accB) + sB * pq;
-        sA = __dp4a(a, 0x01010101u, sA);
-        sB = __dp4a(b, 0x01010101u, sB);
-        P += pq;
-    }
-    return make_uint2(accA | (accB << 16), sA | (sB << 8) | (P << 16));
+    return nib_quads<GChainNib<G, E>::SB / 8>(ch.ab() + k0, ch.pb() + k0);
 }
 // lo then hi: acc = acc_lo + acc_hi + X_lo * P_hi for both weights (no carry between the 16-bit
 // halves: the joined forms fit 16 bits), the byte sums and P add field-wise
@@ -155,6 +160,7 @@ __device__ __forceinline__ void bt_spread_load(const GChainNib<G, E>& ch, int Ls
 template <int G, int E>
 __device__ __forceinline__ int32_t gchain_eval_nib(const GChainNib<G, E>& ch, int l, int gbase, int n,
                                                    int32_t d, uint32_t tAB, uint32_t tP, int quad) {
+    using C = GChainNib<G, E>;
     const uint32_t iP = gscan<G>(tP);
     const uint32_t iAB = gscan<G>(tAB);
     const int32_t Pb = (int32_t)(iP - tP);
@@ -179,7 +185,7 @@ __device__ __forceinline__ int32_t gchain_eval_nib(const GChainNib<G, E>& ch, in
     const uint2* srow = ch.sum() + l;
     uint32_t acc = 0, xb = 0;
 #pragma unroll
-    for (int b = 0; b < E / 16; ++b) {
+    for (int b = 0; b < C::NSB; ++b) {
         const uint2 s = srow[b * G];
         acc = __dp2a_lo(s.x, asel, acc) + xb * (s.y >> 16);
         xb = __dp4a(s.y, xsel, xb);

@@ -433,7 +433,8 @@ def test_balanced_schedule_every_chain(lib, problem, n, chains, steps):
 
 
 # The nibble layout with sub-block summaries (csrc/sa_nib.cuh): CDD with alpha, beta <= 15 and
-# pmax * max(alpha, beta) * 120 < 2^16 at G = 8, E = 128 (n in (512, 1024]).  Every move of <= 4
+# pmax * max(alpha, beta) * 120 < 2^16 at G = 8, E = 128 (n in (512, 1024]; 16-position sub-blocks)
+# or E = 64 (n in (256, 512]; 8-position sub-blocks).  Every move of <= 4
 # positions (insertion keeps the byte rows at this layout: the same check covers it), traced chain
 # by chain against the oracle, and the same run with the byte-row layout
 # (CDD_SA_NO_NIB=1) must give the identical trace.  The instances put the 16-bit sub-block forms
@@ -447,6 +448,10 @@ NIB = [
     (513, dict(p=(1, 20), alpha=(0, 0), beta=(1, 15), h=0.0)),
     (1024, dict(p=(1, 20), alpha=(1, 15), beta=(0, 0), h=1.2)),
     (1024, dict(p=(36, 36), alpha=(15, 15), beta=(15, 15), h=0.5)),
+    # 8-position sub-blocks at E = 64 (n in (256, 512])
+    (500, dict(p=(1, 20), alpha=(1, 10), beta=(1, 15), h=0.6)),
+    (257, dict(p=(30, 36), alpha=(0, 15), beta=(0, 15), h=0.3)),
+    (512, dict(p=(1, 36), alpha=(15, 15), beta=(15, 15), h=1.1)),
 ]
 
 
@@ -457,7 +462,7 @@ def test_nibble_layout_trace_parity(lib, n, kw, move, pert):
     chains, steps, seed = 48, 150, 77 + n
     ins, res, (pen, perm, gid), pr, p, T0 = _run_both(lib, inst, "cdd", chains, steps, seed, samples=300,
                                                      move=move, pert=pert, lanes=8)
-    assert lib.sa_layout(ins, chains, lanes=8) == (8, 128) and ins.query()["small_weights"]
+    assert lib.sa_layout(ins, chains, lanes=8) == (8, 128 if n > 512 else 64) and ins.query()["small_weights"]
     tr = res["trace"].cpu().numpy()
     for c in range(chains):
         ref = oracle.sa_chain(pr, p, T0, c, trace=True)
