@@ -169,7 +169,7 @@ __global__ void t0_reduce_kernel(const int64_t* __restrict__ Z, int64_t N, doubl
 // resident CTAs the register budget is sized for: as many as shared memory admits, at most
 // CDD_SAG_MIN_BLOCKS (UCDDCP at E = 64 holds 58 KB of chains per CTA -> 3)
 // the chain layout of a group-kernel variant: MV = 2 is the nibble layout with sub-block
-// summaries (sa_nib.cuh; CDD, moves of <= 4 positions, G = 8, E = 128)
+// summaries (sa_nib.cuh; CDD, moves of <= 4 positions, G = 8, E = 128 or 64)
 template <int G, int E, bool UCD, int MV>
 struct SagChainT {
     using type = GChain<G, E, UCD>;

@@ -1,6 +1,6 @@
 // sa_nib.cuh -- the CDD chain layout of the headline SA configuration for instances with small
 // weights: 4-bit alpha and beta packed in one byte per position, P in a byte row, and a cached
-// summary per 16-position sub-block of every lane row.
+// summary per sub-block (16 positions at E = 128, 8 at E = 64) of every lane row.
 //
 // Why: at n = 1000 (G = 8 lanes x E = 128 positions) the group kernel's per-step pass streams the
 // whole chain (5 instructions per 4 positions, a third of the step), and the boundary row's level
