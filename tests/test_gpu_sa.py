@@ -484,13 +484,18 @@ def test_nibble_layout_full_grid_and_balanced(lib):
     # the oracle, round robin over more chains than resident slots and the balanced schedule
     import torch
 
-    inst = gen.cdd_instance(1000, 3, 0.6)
+    for n, chain_counts in ((1000, (70000, 73040)), (500, (16208, 30000))):
+        _full_grid(lib, torch, n, chain_counts)
+
+
+def _full_grid(lib, torch, n, chain_counts):
+    inst = gen.cdd_instance(n, 3, 0.6)
     pr = _prob(inst)
-    for chains in (70000, 73040):
+    for chains in chain_counts:
         ins = lib.Instance.from_gen(inst)
         res = lib.sa_run(ins, chains, 40, T0=500.0, seed=11, chain_best=True, chain_final=True)
         torch.cuda.synchronize()
-        assert lib.sa_layout(ins, chains) == (8, 128)
+        assert lib.sa_layout(ins, chains) == (8, 128 if n > 512 else 64)
         cb, cf = res["chain_best"].cpu().numpy(), res["chain_final"].cpu().numpy()
         p = oracle.sa_params(chains=1, steps=40, seed=11)
         for c in list(range(0, chains, 997)) + [chains - 1]:
